@@ -1,0 +1,189 @@
+/*
+ * up.h -- C ABI of libup.so, the B200 (sm_100a) hot path of UltraPrecise
+ * (Li, Xiao, Yu, Lee, Zhang, ICDE 2024; /root/reference/PAPER.md, cited as
+ * "P:L<line> §<section>").
+ *
+ * What it computes: column-at-a-time evaluation of fixed-point DECIMAL(p,s)
+ * expressions (+ - * / % and unary -, over columns c1..cK and decimal
+ * literals) and the exact SUM over them, RSA-style modular exponentiation,
+ * and a fixed-point Taylor sine.  Semantics and typing: §II,
+ * P:L1028-1080 §III-B3, readings Q1-Q16 in DESIGN.md.
+ *
+ * Conventions (all entry points):
+ *  - Every call returns up_status; nothing throws across the ABI.  On error
+ *    up_last_error() returns a thread-local message.
+ *  - Pointers named d_* and the up_column.data field are DEVICE pointers;
+ *    everything else is host memory.  Device memory passed in is CALLER-owned
+ *    (e.g. torch tensors) and never freed by the library; the ctx owns only
+ *    its kernel cache, workspaces and staging buffers.
+ *  - `stream` is a cudaStream_t (NULL = legacy default stream).  All work is
+ *    ordered on it; calls return without synchronising unless stated.
+ *  - Data-dependent arithmetic faults (declared-type overflow, divide by
+ *    zero, out-of-range input) never abort a kernel: they set a sticky device
+ *    flag that up_check() reads (values of the affected rows are unspecified).
+ *  - One ctx per host thread / stream (its SUM workspace is not shared-safe).
+ */
+#ifndef UP_H
+#define UP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    UP_OK = 0,
+    UP_E_INVAL = 1,        /* bad argument, bad expression, % on non-integers */
+    UP_E_RANGE = 2,        /* input value does not fit its DECIMAL(p,s) */
+    UP_E_OVERFLOW = 3,     /* a value exceeded its inferred type (reading Q5: only / can) */
+    UP_E_DIVZERO = 4,      /* division or modulo by zero (reading Q6) */
+    UP_E_NOMEM = 5,
+    UP_E_CUDA = 6,         /* CUDA runtime / driver error */
+    UP_E_NVRTC = 7,        /* kernel specialisation (JIT) failed */
+    UP_E_UNSUPPORTED = 8   /* valid request outside what this build implements */
+} up_status;
+
+const char *up_last_error(void);
+
+typedef struct up_ctx up_ctx;
+
+/* Create a context bound to CUDA device `device` (makes it current). */
+up_status up_ctx_create(int device, up_ctx **out);
+up_status up_ctx_destroy(up_ctx *ctx);
+
+/*
+ * A DECIMAL(p,s) column of n rows as `limbs` limb planes (SURVEY §8a layout):
+ * data[j*ld + i] is limb j (little-endian, 32-bit) of row i's mantissa in
+ * TWO'S COMPLEMENT, value = mantissa * 10^-s (Eq. 1).  ld >= n is a
+ * multiple of 4 and data is 16-byte aligned.  limbs must equal up_limbs(p).
+ * Rows n..ld-1 are padding and are never read as values.
+ */
+typedef struct {
+    int64_t n, ld;
+    int32_t p, s, limbs, reserved;
+    uint32_t *data;
+} up_column;
+
+/* Limb count L = min{L : 10^p <= 2^(32L-1)} (reading Q1 of P:L821-837 vs
+ * reproduces 18/38/76/153/307 <-> 2/4/8/16/32). */
+int32_t up_limbs(int32_t p);
+/* ld for n rows (n rounded up to a multiple of 4). */
+int64_t up_ld(int64_t n);
+/* SUM result precision p + ceil(log10 N), N = n_global (reading Q9). */
+int32_t up_sum_precision(int32_t p, int64_t n_global);
+
+/*
+ * Column ingestion (row a3).  Sign-magnitude binary input: row i's magnitude
+ * is mag[i*mag_words .. +mag_words) (little-endian uint32), its sign neg[i]
+ * (nonzero = negative; NULL = all non-negative).  dst must be preset by the
+ * caller: n, ld, p, s, limbs, data (device, limbs*ld uint32).  A magnitude
+ * >= 10^p sets the RANGE flag (see up_check).
+ *   _host_bin: mag/neg are HOST pointers (pinned for async copies); they are
+ *              staged through ctx-owned device memory on `stream`; the call
+ *              returns after the host buffers may be reused (it synchronises
+ *              the stream before returning).
+ *   _device_bin: mag/neg are DEVICE pointers (e.g. from the generator).
+ *   _host: decimal strings "[-]ddd[.ddd]" (at most s fraction digits, else
+ *              UP_E_RANGE); parsed on the host, then as _host_bin.
+ */
+up_status up_column_from_host_bin(up_ctx *ctx, const uint32_t *mag, int32_t mag_words,
+                                  const uint8_t *neg, up_column *dst, void *stream);
+up_status up_column_from_device_bin(up_ctx *ctx, const uint32_t *d_mag, int32_t mag_words,
+                                    const uint8_t *d_neg, up_column *dst, void *stream);
+up_status up_column_from_host(up_ctx *ctx, const char *const *decimals, up_column *dst, void *stream);
+/* Column to host as sign-magnitude: mag (n x col->limbs words), neg (n bytes).
+ * Synchronises the stream. */
+up_status up_column_to_host_bin(up_ctx *ctx, const up_column *col, uint32_t *mag, uint8_t *neg,
+                                void *stream);
+
+/* Result type of expr over the columns (§III-B3). */
+up_status up_expr_type(up_ctx *ctx, const char *expr, const up_column *cols, int ncols,
+                       int32_t *p, int32_t *s);
+
+/*
+ * Evaluate expr for every row (rows a1-a7, a12): out must be caller-allocated
+ * with up_expr_type's (p,s), limbs = up_limbs(p), n = cols[0].n.  The first
+ * call for an (expr, column types) pair specialises and JIT-compiles a fused
+ * kernel for sm_100a (row a2, §III-B); later calls hit the cache.
+ */
+up_status up_eval_expr(up_ctx *ctx, const char *expr, const up_column *cols, int ncols,
+                       up_column *out, void *stream);
+
+/*
+ * SELECT SUM(expr) over this shard's rows (row a11), fused with evaluation.
+ * The result type is DECIMAL(p_expr + ceil(log10 n_global), s_expr) with
+ * LA = up_limbs(that p) limbs (query with up_sum_type).  d_partial receives LA
+ * two's-complement limbs (device).  n_global = rows over all shards (typing
+ * only; 0 means cols[0].n).  One kernel launch.
+ */
+up_status up_sum_type(up_ctx *ctx, const char *expr, const up_column *cols, int ncols,
+                      int64_t n_global, int32_t *p, int32_t *s, int32_t *la);
+up_status up_sum_expr(up_ctx *ctx, const char *expr, const up_column *cols, int ncols,
+                      int64_t n_global, uint32_t *d_partial, void *stream);
+/* SUM of one column: up_sum_expr(ctx, "c1", col, 1, ...). */
+up_status up_sum(up_ctx *ctx, const up_column *col, int64_t n_global, uint32_t *d_partial, void *stream);
+
+/*
+ * Exact combine of nranks SUM partials (row a13): d_partials holds nranks x la
+ * two's-complement limbs (device, rank-major, e.g. an NCCL all-gather
+ * output); d_out receives their sum in la limbs.  One kernel launch.
+ */
+up_status up_sum_combine(up_ctx *ctx, const uint32_t *d_partials, int32_t nranks, int32_t la,
+                         uint32_t *d_out, void *stream);
+
+/*
+ * x^e mod N per row (row a8; Query 4 P:L2124-2154 generalised to any e).
+ * base: s == 0, values >= 0 (a negative value sets INVAL); values >= N are
+ * reduced mod N first.  exponent, modulus: decimal strings, modulus odd and
+ * > 1 (even moduli: UP_E_UNSUPPORTED).  out: DECIMAL(digits(N), 0),
+ * caller-allocated (p = number of decimal digits of N).  N is converted and
+ * its Montgomery constants are derived at specialisation time.
+ * up_modexp_sum: fused SUM of the results into d_partial, type
+ * DECIMAL(digits(N) + ceil(log10 n_global), 0) (query with up_modexp_sum_type).
+ */
+up_status up_modexp(up_ctx *ctx, const up_column *base, const char *exponent, const char *modulus,
+                    up_column *out, void *stream);
+up_status up_modexp_sum_type(up_ctx *ctx, const char *modulus, int64_t n_global,
+                             int32_t *p, int32_t *la);
+up_status up_modexp_sum(up_ctx *ctx, const up_column *base, const char *exponent, const char *modulus,
+                        int64_t n_global, uint32_t *d_partial, void *stream);
+
+/*
+ * Fixed-point Taylor sine sin_P(x) per row (row a9, from
+ * Query 5 P:L2197-2249): x DECIMAL(p,s) with s <= 9, p - s <= 1 (|x| < 10),
+ * t_1 = |m_x| 10^(P-s), t_{k+1} = floor(t_k m_x^2 / (10^(2s) (2k)(2k+1))),
+ * result sign(m_x) * sum_k (-1)^(k-1) t_k, type DECIMAL(P+1, P).
+ * up_sin_taylor: out caller-allocated DECIMAL(P+1,P).
+ * up_sin_taylor_sum: fused SUM, type DECIMAL(P+1+ceil(log10 n_global), P).
+ */
+up_status up_sin_taylor(up_ctx *ctx, const up_column *x, int32_t P, up_column *out, void *stream);
+up_status up_sin_taylor_sum(up_ctx *ctx, const up_column *x, int32_t P, int64_t n_global,
+                            uint32_t *d_partial, void *stream);
+
+/* Synchronise the stream and read + clear the sticky device flags:
+ * UP_E_OVERFLOW / UP_E_DIVZERO / UP_E_RANGE / UP_E_INVAL (first in that order). */
+up_status up_check(up_ctx *ctx, void *stream);
+
+/* Format `limbs` two's-complement limbs (HOST memory) at scale s as the
+ * canonical "[-]int.frac" string (exactly s fraction digits, no "-0"). */
+up_status up_format_decimal(const uint32_t *limbs, int32_t nlimbs, int32_t s, char *buf, size_t len);
+
+/* Number of kernels this ctx has launched (evidence for gpu_launches). */
+uint64_t up_launch_count(up_ctx *ctx);
+/* Milliseconds spent in NVRTC specialisation so far (excluded from timing). */
+double up_jit_ms(up_ctx *ctx);
+
+/* Diagnostics (no GPU needed).  up_gen_source: the CUDA source the
+ * specialiser emits for variant "sum" or "eval" (cols supply types only).
+ * up_nvrtc_compile: NVRTC-compile a source for sm_100a (ptxas -v log into
+ * `log`; cubin written to cubin_path if non-NULL). */
+up_status up_gen_source(const char *variant, const char *expr, const up_column *cols, int ncols,
+                        int64_t n_global, char *buf, size_t len);
+up_status up_nvrtc_compile(const char *src, const char *cubin_path, char *log, size_t len);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* UP_H */

@@ -1,0 +1,32 @@
+// codegen.h -- kernel specialisation (row a2).
+#pragma once
+#include <string>
+#include <vector>
+
+#include "expr.h"
+
+namespace uph {
+
+struct GenOpts {
+    bool sum = false;   // fused SUM (true) or per-row column output (false)
+    int LA = 0;         // SUM limbs
+};
+
+struct GenInfo {
+    int rows_per_thread = 1;
+    int ws_slots = 0;
+};
+
+std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, const GenOpts &opt, GenInfo &info);
+
+// modexp / sin_taylor specialisations (special.cpp)
+struct ModexpPlan {
+    int n = 0;          // modulus limbs
+    int Lb = 0;         // base column limbs
+    int Lout = 0;       // output limbs
+    int LA = 0;         // SUM limbs (sum variant)
+};
+std::string gen_modexp_kernel(const HBig &N, const HBig &e, const ModexpPlan &plan, bool sum, std::string &err);
+std::string gen_sin_kernel(int P, int p, int s, int Lx, int Lout, int LA, bool sum, int &lanes_per_row, std::string &err);
+
+}  // namespace uph

@@ -1,0 +1,116 @@
+// kernels.cu -- static (nvcc, sm_100a) kernels of libup: column codec (row a3
+// ingestion / row a12 read-back) and the exact multi-rank combine (row a13).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "up_dev.cuh"
+
+using up::u32;
+using up::u64;
+
+namespace {
+
+// sign-magnitude rows (n x W words, neg bytes) -> L two's-complement planes.
+// One thread per row; planes written coalesced.  |mag| >= 10^p sets F_RANGE
+// (bound = 10^p in L limbs, a DECIMAL(p,s) holds |m| < 10^p, Eq. 1).
+__global__ void __launch_bounds__(256) k_from_bin(const u32 *__restrict__ mag, int W, const uint8_t *__restrict__ neg,
+                                                  long long n, const u32 *__restrict__ bound, int L,
+                                                  u32 *__restrict__ out, long long ld, u32 *flags) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    u32 fl = 0;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const u32 *m = mag + i * W;
+        // range check, most significant limb first
+        int cmp = 0;   // -1: m < bound, +1: m >= bound decided
+        for (int j = (W > L ? W : L) - 1; j >= 0 && cmp == 0; --j) {
+            const u32 a = j < W ? m[j] : 0u, b = j < L ? bound[j] : 0u;
+            if (a != b) cmp = a < b ? -1 : 1;
+        }
+        if (cmp >= 0) fl |= up::F_RANGE;
+        const u32 ng = (neg && neg[i]) ? 1u : 0u;
+        const u32 mask = 0u - ng;
+        u64 carry = ng;
+        for (int j = 0; j < L; ++j) {
+            const u64 t = (u64)((j < W ? m[j] : 0u) ^ mask) + carry;
+            out[(long long)j * ld + i] = (u32)t;
+            carry = t >> 32;
+        }
+    }
+    if (fl) atomicOr(flags, fl);
+}
+
+// L two's-complement planes -> sign-magnitude rows (n x L words, neg bytes)
+__global__ void __launch_bounds__(256) k_to_bin(const u32 *__restrict__ planes, int L, long long ld, long long n,
+                                                u32 *__restrict__ mag, uint8_t *__restrict__ neg) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const u32 ng = planes[(long long)(L - 1) * ld + i] >> 31;
+        const u32 mask = 0u - ng;
+        u64 carry = ng;
+        for (int j = 0; j < L; ++j) {
+            const u64 t = (u64)(planes[(long long)j * ld + i] ^ mask) + carry;
+            mag[i * L + j] = (u32)t;
+            carry = t >> 32;
+        }
+        neg[i] = (uint8_t)ng;
+    }
+}
+
+// out = sum of nranks la-limb two's-complement partials, mod 2^(32 la), in
+// rank order (exact; order only matters for readability -- integer sums
+// commute).  One block: limb-parallel 64-bit column sums, then one carry pass.
+__global__ void __launch_bounds__(1024) k_combine(const u32 *__restrict__ parts, int nranks, int la,
+                                                  u32 *__restrict__ out) {
+    extern __shared__ u64 col[];
+    for (int j = threadIdx.x; j < la; j += blockDim.x) {
+        u64 t = 0;
+        for (int r = 0; r < nranks; ++r) t += parts[(long long)r * la + j];
+        col[j] = t;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        u64 carry = 0;
+        for (int j = 0; j < la; ++j) {
+            const u64 t = (col[j] & 0xffffffffull) + carry;
+            out[j] = (u32)t;
+            carry = (t >> 32) + (col[j] >> 32);
+        }
+    }
+}
+
+int grid_for(long long n, int threads) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    long long want = (n + threads - 1) / threads;
+    long long cap = (long long)sms * 8;
+    return (int)(want < 1 ? 1 : (want < cap ? want : cap));
+}
+
+}  // namespace
+
+extern "C" {
+
+cudaError_t upk_launch_from_bin(const uint32_t *mag, int W, const uint8_t *neg, long long n, const uint32_t *bound,
+                                int L, uint32_t *out, long long ld, uint32_t *flags, cudaStream_t st) {
+    k_from_bin<<<grid_for(n, 256), 256, 0, st>>>(mag, W, neg, n, bound, L, out, ld, flags);
+    return cudaGetLastError();
+}
+
+cudaError_t upk_launch_to_bin(const uint32_t *planes, int L, long long ld, long long n, uint32_t *mag, uint8_t *neg,
+                              cudaStream_t st) {
+    k_to_bin<<<grid_for(n, 256), 256, 0, st>>>(planes, L, ld, n, mag, neg);
+    return cudaGetLastError();
+}
+
+cudaError_t upk_launch_combine(const uint32_t *partials, int nranks, int la, uint32_t *out, cudaStream_t st) {
+    const size_t smem = sizeof(u64) * (size_t)la;
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(k_combine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    k_combine<<<1, 1024, smem, st>>>(partials, nranks, la, out);
+    return cudaGetLastError();
+}
+
+}  // extern "C"

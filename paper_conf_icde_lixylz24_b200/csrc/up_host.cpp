@@ -1,0 +1,606 @@
+// up_host.cpp -- the C ABI of libup.so (include/up.h): context, NVRTC
+// specialisation + kernel cache (row a2), launches, column codec, combine.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <nvrtc.h>
+
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <fstream>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "../../include/up.h"
+#include "codegen.h"
+#include "expr.h"
+#include "hbig.h"
+#include "up_embed.inc"   // k_up_dev_src, k_up_kparams_src (generated from up_dev.cuh / up_kparams.h)
+#include "up_kparams.h"
+
+using namespace uph;
+
+// ---------------------------------------------------------------- static kernels (kernels.cu)
+extern "C" {
+cudaError_t upk_launch_from_bin(const uint32_t *mag, int W, const uint8_t *neg, long long n, const uint32_t *bound,
+                                int L, uint32_t *out, long long ld, uint32_t *flags, cudaStream_t st);
+cudaError_t upk_launch_to_bin(const uint32_t *planes, int L, long long ld, long long n, uint32_t *mag, uint8_t *neg,
+                              cudaStream_t st);
+cudaError_t upk_launch_combine(const uint32_t *partials, int nranks, int la, uint32_t *out, cudaStream_t st);
+}
+
+namespace {
+
+thread_local std::string g_err;
+
+// Driver API entry points fetched through the runtime, so libup.so has no
+// link-time dependency on libcuda.so.1 (it loads on GPU-less build hosts).
+struct Drv {
+    CUresult (*ModuleLoadData)(CUmodule *, const void *) = nullptr;
+    CUresult (*ModuleGetFunction)(CUfunction *, CUmodule, const char *) = nullptr;
+    CUresult (*ModuleUnload)(CUmodule) = nullptr;
+    CUresult (*LaunchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                             CUstream, void **, void **) = nullptr;
+    CUresult (*OccupancyMaxActiveBlocksPerMultiprocessor)(int *, CUfunction, int, size_t) = nullptr;
+    CUresult (*GetErrorString)(CUresult, const char **) = nullptr;
+    bool ok = false;
+} drv;
+
+cudaError_t load_drv() {
+    if (drv.ok) return cudaSuccess;
+    cudaDriverEntryPointQueryResult q;
+#define UP_ENTRY(name, field)                                                                            \
+    do {                                                                                                 \
+        cudaError_t e = cudaGetDriverEntryPoint(name, (void **)&drv.field, cudaEnableDefault, &q);      \
+        if (e != cudaSuccess) return e;                                                                  \
+        if (q != cudaDriverEntryPointSuccess || !drv.field) return cudaErrorSymbolNotFound;              \
+    } while (0)
+    UP_ENTRY("cuModuleLoadData", ModuleLoadData);
+    UP_ENTRY("cuModuleGetFunction", ModuleGetFunction);
+    UP_ENTRY("cuModuleUnload", ModuleUnload);
+    UP_ENTRY("cuLaunchKernel", LaunchKernel);
+    UP_ENTRY("cuOccupancyMaxActiveBlocksPerMultiprocessor", OccupancyMaxActiveBlocksPerMultiprocessor);
+    UP_ENTRY("cuGetErrorString", GetErrorString);
+#undef UP_ENTRY
+    drv.ok = true;
+    return cudaSuccess;
+}
+
+up_status fail(up_status st, const char *fmt, ...) {
+    char buf[2048];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return st;
+}
+
+#define CUDA_TRY(x)                                                                          \
+    do {                                                                                     \
+        cudaError_t e_ = (x);                                                                \
+        if (e_ != cudaSuccess) return fail(UP_E_CUDA, "%s: %s", #x, cudaGetErrorString(e_)); \
+    } while (0)
+#define CU_TRY(x)                                                                         \
+    do {                                                                                  \
+        CUresult e_ = (x);                                                                \
+        if (e_ != CUDA_SUCCESS) {                                                         \
+            const char *s_ = nullptr;                                                     \
+            if (drv.GetErrorString) drv.GetErrorString(e_, &s_);                          \
+            return fail(UP_E_CUDA, "%s: %s", #x, s_ ? s_ : "?");                          \
+        }                                                                                 \
+    } while (0)
+
+constexpr int kThreads = 256;
+constexpr int kWsSlots = 1 << 16;
+
+struct JitKernel {
+    CUmodule mod = nullptr;
+    CUfunction fn = nullptr;
+    int rows_per_thread = 1;
+    int ws_slots = 0;
+    int blocks_per_sm = 1;
+    int threads = kThreads;
+    std::string src;
+};
+
+}  // namespace
+
+struct up_ctx {
+    int device = 0;
+    int num_sms = 148;
+    unsigned long long *d_ws = nullptr;   // SUM slots
+    uint32_t *d_ticket = nullptr;
+    uint32_t *d_flags = nullptr;
+    void *d_stage = nullptr;
+    size_t stage_bytes = 0;
+    std::map<int, uint32_t *> pow10_dev;  // 10^p magnitude in up_limbs(p) limbs
+    std::unordered_map<std::string, std::unique_ptr<JitKernel>> by_src;
+    std::unordered_map<std::string, JitKernel *> by_key;
+    uint64_t launches = 0;
+    double jit_ms = 0.0;
+    std::mutex mu;
+};
+
+namespace {
+
+up_status ensure_stage(up_ctx *c, size_t bytes, cudaStream_t st) {
+    if (bytes <= c->stage_bytes) return UP_OK;
+    if (c->d_stage) {
+        CUDA_TRY(cudaStreamSynchronize(st));
+        CUDA_TRY(cudaFree(c->d_stage));
+        c->d_stage = nullptr;
+    }
+    size_t nb = std::max(bytes, c->stage_bytes * 2);
+    CUDA_TRY(cudaMalloc(&c->d_stage, nb));
+    c->stage_bytes = nb;
+    return UP_OK;
+}
+
+up_status pow10_device(up_ctx *c, int p, const uint32_t **out) {
+    auto it = c->pow10_dev.find(p);
+    if (it != c->pow10_dev.end()) { *out = it->second; return UP_OK; }
+    const int L = limbs_for_precision(p);
+    std::vector<uint32_t> w = HBig::pow10(p).twos(L, false);
+    uint32_t *d = nullptr;
+    CUDA_TRY(cudaMalloc(&d, sizeof(uint32_t) * (size_t)L));
+    CUDA_TRY(cudaMemcpy(d, w.data(), sizeof(uint32_t) * (size_t)L, cudaMemcpyHostToDevice));
+    c->pow10_dev[p] = d;
+    *out = d;
+    return UP_OK;
+}
+
+up_status check_column(const up_column *col, const char *what) {
+    if (!col) return fail(UP_E_INVAL, "%s: null column", what);
+    if (col->p < 1 || col->s < 0) return fail(UP_E_INVAL, "%s: bad DECIMAL(%d,%d)", what, col->p, col->s);
+    if (col->limbs != limbs_for_precision(col->p))
+        return fail(UP_E_INVAL, "%s: limbs %d != up_limbs(%d) = %d", what, col->limbs, col->p, limbs_for_precision(col->p));
+    if (col->n < 0 || col->ld < col->n || (col->ld & 3)) return fail(UP_E_INVAL, "%s: bad n/ld (%lld/%lld)", what, (long long)col->n, (long long)col->ld);
+    if (col->n > 0 && (!col->data || ((uintptr_t)col->data & 15))) return fail(UP_E_INVAL, "%s: data must be 16-byte aligned device memory", what);
+    if (col->n >= (1ll << 32)) return fail(UP_E_UNSUPPORTED, "%s: more than 2^32-1 rows per call", what);
+    return UP_OK;
+}
+
+const char *kNvrtcOpts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-default-device", "-lineinfo", "-DNDEBUG"};
+
+up_status compile(up_ctx *c, const std::string &src, JitKernel **out) {
+    auto it = c->by_src.find(src);
+    if (it != c->by_src.end()) { *out = it->second.get(); return UP_OK; }
+    auto t0 = std::chrono::steady_clock::now();
+    if (const char *dump = getenv("UP_DUMP_DIR")) {
+        std::string path = std::string(dump) + "/upk_" + std::to_string(c->by_src.size()) + ".cu";
+        std::ofstream(path) << src;
+    }
+    nvrtcProgram prog;
+    const char *hdrs[2] = {k_up_dev_src, k_up_kparams_src};
+    const char *names[2] = {"up_dev.cuh", "up_kparams.h"};
+    if (nvrtcCreateProgram(&prog, src.c_str(), "upk.cu", 2, hdrs, names) != NVRTC_SUCCESS)
+        return fail(UP_E_NVRTC, "nvrtcCreateProgram failed");
+    nvrtcResult r = nvrtcCompileProgram(prog, (int)(sizeof kNvrtcOpts / sizeof kNvrtcOpts[0]), kNvrtcOpts);
+    if (r != NVRTC_SUCCESS) {
+        size_t ls = 0;
+        nvrtcGetProgramLogSize(prog, &ls);
+        std::string log(ls, '\0');
+        nvrtcGetProgramLog(prog, &log[0]);
+        nvrtcDestroyProgram(&prog);
+        return fail(UP_E_NVRTC, "NVRTC: %s\n%s", nvrtcGetErrorString(r), log.substr(0, 1500).c_str());
+    }
+    size_t cs = 0;
+    nvrtcGetCUBINSize(prog, &cs);
+    std::vector<char> cubin(cs);
+    nvrtcGetCUBIN(prog, cubin.data());
+    nvrtcDestroyProgram(&prog);
+    auto k = std::make_unique<JitKernel>();
+    CU_TRY(drv.ModuleLoadData(&k->mod, cubin.data()));
+    CU_TRY(drv.ModuleGetFunction(&k->fn, k->mod, "upk"));
+    int nb = 0;
+    CU_TRY(drv.OccupancyMaxActiveBlocksPerMultiprocessor(&nb, k->fn, kThreads, 0));
+    k->blocks_per_sm = std::max(1, nb);
+    k->src = src;
+    c->jit_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    *out = k.get();
+    c->by_src[src] = std::move(k);
+    return UP_OK;
+}
+
+struct Typed {
+    std::unique_ptr<Node> root;
+    std::vector<ColType> types;
+};
+
+up_status type_expr(const char *expr, const up_column *cols, int ncols, Typed &t) {
+    if (!expr) return fail(UP_E_INVAL, "null expression");
+    if (ncols < 0 || ncols > UP_MAX_COLS) return fail(UP_E_UNSUPPORTED, "at most %d columns", UP_MAX_COLS);
+    for (int i = 0; i < ncols; ++i) {
+        if (cols[i].p < 1 || cols[i].s < 0 || cols[i].limbs != limbs_for_precision(cols[i].p))
+            return fail(UP_E_INVAL, "column %d: bad type/limbs", i + 1);
+        t.types.push_back({cols[i].p, cols[i].s, cols[i].limbs});
+    }
+    std::string err;
+    t.root = parse_expr(expr, ncols, err);
+    if (!t.root) return fail(UP_E_INVAL, "expression '%s': %s", expr, err.c_str());
+    if (type_tree(t.root.get(), t.types, err)) return fail(UP_E_INVAL, "expression '%s': %s", expr, err.c_str());
+    return UP_OK;
+}
+
+std::string key_of(const char *tag, const char *expr, const up_column *cols, int ncols, int extra) {
+    std::string k = tag;
+    k += '|';
+    k += expr;
+    for (int i = 0; i < ncols; ++i) k += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
+    k += "|" + std::to_string(extra);
+    return k;
+}
+
+up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream_t st) {
+    long long per_block = (long long)k->threads * k->rows_per_thread;
+    long long want = (n + per_block - 1) / per_block;
+    long long cap = (long long)k->blocks_per_sm * c->num_sms;
+    int grid = (int)std::max(1ll, std::min(want, cap));
+    void *args[] = {&P};
+    CU_TRY(drv.LaunchKernel(k->fn, grid, 1, 1, k->threads, 1, 1, 0, (CUstream)st, args, nullptr));
+    c->launches++;
+    return UP_OK;
+}
+
+up_status expr_kernel(up_ctx *c, const char *expr, const up_column *cols, int ncols, bool sum, long long n_global,
+                      JitKernel **out, int *LA_out, Node **root_out, Typed &t) {
+    up_status s = type_expr(expr, cols, ncols, t);
+    if (s) return s;
+    const int ps = sum_precision(t.root->p, n_global);
+    const int LA = sum ? limbs_for_precision(ps) : 0;
+    if (LA_out) *LA_out = LA;
+    if (root_out) *root_out = t.root.get();
+    std::string key = key_of(sum ? "sum" : "eval", expr, cols, ncols, LA);
+    auto it = c->by_key.find(key);
+    if (it != c->by_key.end()) { *out = it->second; return UP_OK; }
+    GenOpts o;
+    o.sum = sum;
+    o.LA = LA;
+    GenInfo info;
+    std::string src = gen_expr_kernel(t.root.get(), t.types, o, info);
+    if (sum && info.ws_slots > kWsSlots) return fail(UP_E_UNSUPPORTED, "SUM too wide (%d slots)", info.ws_slots);
+    JitKernel *k = nullptr;
+    s = compile(c, src, &k);
+    if (s) return s;
+    k->rows_per_thread = info.rows_per_thread;
+    k->ws_slots = info.ws_slots;
+    c->by_key[key] = k;
+    *out = k;
+    return UP_OK;
+}
+
+void fill_cols(up_kparams &P, const up_column *cols, int ncols) {
+    memset(&P, 0, sizeof P);
+    for (int i = 0; i < ncols; ++i) {
+        P.col[i] = cols[i].data;
+        P.ld[i] = cols[i].ld;
+    }
+    P.n = ncols ? cols[0].n : 0;
+}
+
+}  // namespace
+
+// ====================================================================== C ABI
+extern "C" {
+
+const char *up_last_error(void) { return g_err.c_str(); }
+
+int32_t up_limbs(int32_t p) { return limbs_for_precision(p); }
+int64_t up_ld(int64_t n) { return (n + 3) & ~3ll; }
+int32_t up_sum_precision(int32_t p, int64_t n_global) { return sum_precision(p, n_global); }
+
+up_status up_ctx_create(int device, up_ctx **out) {
+    if (!out) return fail(UP_E_INVAL, "null out");
+    CUDA_TRY(cudaSetDevice(device));
+    CUDA_TRY(cudaFree(nullptr));   // initialise the primary context (shared with torch)
+    CUDA_TRY(load_drv());
+    auto c = std::make_unique<up_ctx>();
+    c->device = device;
+    CUDA_TRY(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device));
+    CUDA_TRY(cudaMalloc(&c->d_ws, sizeof(unsigned long long) * kWsSlots));
+    CUDA_TRY(cudaMemset(c->d_ws, 0, sizeof(unsigned long long) * kWsSlots));
+    CUDA_TRY(cudaMalloc(&c->d_ticket, 64));
+    CUDA_TRY(cudaMemset(c->d_ticket, 0, 64));
+    CUDA_TRY(cudaMalloc(&c->d_flags, 64));
+    CUDA_TRY(cudaMemset(c->d_flags, 0, 64));
+    CUDA_TRY(cudaDeviceSynchronize());
+    *out = c.release();
+    return UP_OK;
+}
+
+up_status up_ctx_destroy(up_ctx *c) {
+    if (!c) return UP_OK;
+    cudaDeviceSynchronize();
+    for (auto &kv : c->by_src) if (kv.second->mod && drv.ModuleUnload) drv.ModuleUnload(kv.second->mod);
+    for (auto &kv : c->pow10_dev) cudaFree(kv.second);
+    cudaFree(c->d_ws);
+    cudaFree(c->d_ticket);
+    cudaFree(c->d_flags);
+    if (c->d_stage) cudaFree(c->d_stage);
+    delete c;
+    return UP_OK;
+}
+
+uint64_t up_launch_count(up_ctx *c) { return c ? c->launches : 0; }
+double up_jit_ms(up_ctx *c) { return c ? c->jit_ms : 0.0; }
+
+up_status up_column_from_device_bin(up_ctx *c, const uint32_t *d_mag, int32_t W, const uint8_t *d_neg,
+                                    up_column *dst, void *stream) {
+    if (!c) return fail(UP_E_INVAL, "null ctx");
+    if (up_status s = check_column(dst, "dst")) return s;
+    if (W < 1) return fail(UP_E_INVAL, "mag_words must be >= 1");
+    if (dst->n == 0) return UP_OK;
+    std::lock_guard<std::mutex> g(c->mu);
+    const uint32_t *bound = nullptr;
+    if (up_status s = pow10_device(c, dst->p, &bound)) return s;
+    CUDA_TRY(upk_launch_from_bin(d_mag, W, d_neg, dst->n, bound, dst->limbs, dst->data, dst->ld, c->d_flags,
+                                 (cudaStream_t)stream));
+    c->launches++;
+    return UP_OK;
+}
+
+up_status up_column_from_host_bin(up_ctx *c, const uint32_t *mag, int32_t W, const uint8_t *neg, up_column *dst,
+                                  void *stream) {
+    if (!c) return fail(UP_E_INVAL, "null ctx");
+    if (up_status s = check_column(dst, "dst")) return s;
+    if (W < 1) return fail(UP_E_INVAL, "mag_words must be >= 1");
+    if (dst->n == 0) return UP_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    const size_t mb = sizeof(uint32_t) * (size_t)W * (size_t)dst->n, nb = neg ? (size_t)dst->n : 0;
+    const size_t mb_al = (mb + 255) & ~(size_t)255;
+    {
+        std::lock_guard<std::mutex> g(c->mu);
+        if (up_status s = ensure_stage(c, mb_al + nb, st)) return s;
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage, mag, mb, cudaMemcpyHostToDevice, st));
+        if (neg) CUDA_TRY(cudaMemcpyAsync((char *)c->d_stage + mb_al, neg, nb, cudaMemcpyHostToDevice, st));
+    }
+    return up_column_from_device_bin(c, (const uint32_t *)c->d_stage, W,
+                                     neg ? (const uint8_t *)((char *)c->d_stage + mb_al) : nullptr, dst, stream);
+}
+
+up_status up_column_from_host(up_ctx *c, const char *const *decimals, up_column *dst, void *stream) {
+    if (!c || !decimals) return fail(UP_E_INVAL, "null argument");
+    if (up_status s = check_column(dst, "dst")) return s;
+    const long long n = dst->n;
+    const int L = dst->limbs;
+    std::vector<uint32_t> mag((size_t)n * (size_t)L, 0);
+    std::vector<uint8_t> neg((size_t)n, 0);
+    const HBig bound = HBig::pow10(dst->p);
+    for (long long i = 0; i < n; ++i) {
+        const char *p = decimals[i];
+        if (!p) return fail(UP_E_INVAL, "row %lld: null string", i);
+        while (*p == ' ') ++p;
+        bool ng = false;
+        if (*p == '-' || *p == '+') { ng = (*p == '-'); ++p; }
+        std::string ip, fp;
+        while (*p >= '0' && *p <= '9') ip += *p++;
+        if (*p == '.') { ++p; while (*p >= '0' && *p <= '9') fp += *p++; }
+        while (*p == ' ') ++p;
+        if (*p || (ip.empty() && fp.empty())) return fail(UP_E_INVAL, "row %lld: bad decimal '%s'", i, decimals[i]);
+        if ((int)fp.size() > dst->s) return fail(UP_E_RANGE, "row %lld: more than %d fraction digits", i, dst->s);
+        fp.append((size_t)(dst->s - (int)fp.size()), '0');
+        HBig m;
+        HBig::from_dec(ip + fp, m);
+        if (HBig::cmp(m, bound) >= 0) return fail(UP_E_RANGE, "row %lld: '%s' exceeds DECIMAL(%d,%d)", i, decimals[i], dst->p, dst->s);
+        for (int j = 0; j < L; ++j) mag[(size_t)i * L + j] = m.limb((size_t)j);
+        neg[(size_t)i] = (ng && !m.is_zero()) ? 1 : 0;
+    }
+    up_status s = up_column_from_host_bin(c, mag.data(), L, neg.data(), dst, stream);
+    if (s) return s;
+    CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream));   // host temporaries die here
+    return UP_OK;
+}
+
+up_status up_column_to_host_bin(up_ctx *c, const up_column *col, uint32_t *mag, uint8_t *neg, void *stream) {
+    if (!c || !mag || !neg) return fail(UP_E_INVAL, "null argument");
+    if (up_status s = check_column(col, "col")) return s;
+    if (col->n == 0) return UP_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    const size_t mb = sizeof(uint32_t) * (size_t)col->limbs * (size_t)col->n, nb = (size_t)col->n;
+    const size_t mb_al = (mb + 255) & ~(size_t)255;
+    std::lock_guard<std::mutex> g(c->mu);
+    if (up_status s = ensure_stage(c, mb_al + nb, st)) return s;
+    uint32_t *dm = (uint32_t *)c->d_stage;
+    uint8_t *dn = (uint8_t *)c->d_stage + mb_al;
+    CUDA_TRY(upk_launch_to_bin(col->data, col->limbs, col->ld, col->n, dm, dn, st));
+    c->launches++;
+    CUDA_TRY(cudaMemcpyAsync(mag, dm, mb, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaMemcpyAsync(neg, dn, nb, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
+    return UP_OK;
+}
+
+up_status up_expr_type(up_ctx *c, const char *expr, const up_column *cols, int ncols, int32_t *p, int32_t *s) {
+    (void)c;
+    Typed t;
+    if (up_status st = type_expr(expr, cols, ncols, t)) return st;
+    if (p) *p = t.root->p;
+    if (s) *s = t.root->s;
+    return UP_OK;
+}
+
+up_status up_sum_type(up_ctx *c, const char *expr, const up_column *cols, int ncols, int64_t n_global, int32_t *p,
+                      int32_t *s, int32_t *la) {
+    (void)c;
+    Typed t;
+    if (up_status st = type_expr(expr, cols, ncols, t)) return st;
+    const long long N = n_global > 0 ? n_global : (ncols ? cols[0].n : 0);
+    const int ps = sum_precision(t.root->p, N);
+    if (p) *p = ps;
+    if (s) *s = t.root->s;
+    if (la) *la = limbs_for_precision(ps);
+    return UP_OK;
+}
+
+up_status up_eval_expr(up_ctx *c, const char *expr, const up_column *cols, int ncols, up_column *out, void *stream) {
+    if (!c || !cols || ncols < 1) return fail(UP_E_INVAL, "need a ctx and at least one column");
+    for (int i = 0; i < ncols; ++i) {
+        if (up_status s = check_column(&cols[i], "input")) return s;
+        if (cols[i].n != cols[0].n) return fail(UP_E_INVAL, "columns differ in length");
+    }
+    if (up_status s = check_column(out, "out")) return s;
+    std::lock_guard<std::mutex> g(c->mu);
+    JitKernel *k = nullptr;
+    Node *root = nullptr;
+    Typed t;
+    if (up_status s = expr_kernel(c, expr, cols, ncols, false, 0, &k, nullptr, &root, t)) return s;
+    if (out->p != root->p || out->s != root->s || out->n != cols[0].n)
+        return fail(UP_E_INVAL, "out must be DECIMAL(%d,%d) with %lld rows", root->p, root->s, (long long)cols[0].n);
+    up_kparams P;
+    fill_cols(P, cols, ncols);
+    P.out = out->data;
+    P.ld_out = out->ld;
+    P.flags = c->d_flags;
+    if (P.n == 0) return UP_OK;
+    return launch(c, k, P, P.n, (cudaStream_t)stream);
+}
+
+up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int ncols, int64_t n_global,
+                      uint32_t *d_partial, void *stream) {
+    if (!c || !cols || ncols < 1 || !d_partial) return fail(UP_E_INVAL, "need a ctx, columns and d_partial");
+    for (int i = 0; i < ncols; ++i) {
+        if (up_status s = check_column(&cols[i], "input")) return s;
+        if (cols[i].n != cols[0].n) return fail(UP_E_INVAL, "columns differ in length");
+    }
+    std::lock_guard<std::mutex> g(c->mu);
+    JitKernel *k = nullptr;
+    int LA = 0;
+    Typed t;
+    const long long N = n_global > 0 ? n_global : cols[0].n;
+    if (N < cols[0].n) return fail(UP_E_INVAL, "n_global < local rows");
+    if (up_status s = expr_kernel(c, expr, cols, ncols, true, N, &k, &LA, nullptr, t)) return s;
+    up_kparams P;
+    fill_cols(P, cols, ncols);
+    P.ws = c->d_ws;
+    P.ticket = c->d_ticket;
+    P.result = d_partial;
+    P.flags = c->d_flags;
+    return launch(c, k, P, P.n, (cudaStream_t)stream);
+}
+
+up_status up_sum(up_ctx *c, const up_column *col, int64_t n_global, uint32_t *d_partial, void *stream) {
+    return up_sum_expr(c, "c1", col, 1, n_global, d_partial, stream);
+}
+
+up_status up_sum_combine(up_ctx *c, const uint32_t *d_partials, int32_t nranks, int32_t la, uint32_t *d_out,
+                         void *stream) {
+    if (!c || !d_partials || !d_out || nranks < 1 || la < 1) return fail(UP_E_INVAL, "bad combine arguments");
+    CUDA_TRY(upk_launch_combine(d_partials, nranks, la, d_out, (cudaStream_t)stream));
+    c->launches++;
+    return UP_OK;
+}
+
+up_status up_check(up_ctx *c, void *stream) {
+    if (!c) return fail(UP_E_INVAL, "null ctx");
+    CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream));
+    uint32_t f = 0;
+    CUDA_TRY(cudaMemcpy(&f, c->d_flags, sizeof f, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemset(c->d_flags, 0, sizeof f));
+    if (f & 1u) return fail(UP_E_OVERFLOW, "a value exceeded its inferred DECIMAL type");
+    if (f & 2u) return fail(UP_E_DIVZERO, "division or modulo by zero");
+    if (f & 4u) return fail(UP_E_RANGE, "an input value exceeds its DECIMAL(p,s)");
+    if (f & 8u) return fail(UP_E_INVAL, "invalid input value (e.g. negative modexp base)");
+    return UP_OK;
+}
+
+up_status up_format_decimal(const uint32_t *limbs, int32_t nlimbs, int32_t s, char *buf, size_t len) {
+    if (!limbs || nlimbs < 1 || !buf || s < 0) return fail(UP_E_INVAL, "bad format arguments");
+    HBig m;
+    m.w.assign(limbs, limbs + nlimbs);
+    const bool ng = (limbs[nlimbs - 1] >> 31) != 0;
+    if (ng) {   // magnitude of a two's-complement value
+        uint64_t cy = 1;
+        for (auto &x : m.w) { uint64_t t = (uint64_t)(~x) + cy; x = (uint32_t)t; cy = t >> 32; }
+    }
+    m.trim();
+    std::string d = m.to_dec();
+    std::string out = (ng && !m.is_zero()) ? "-" : "";
+    if (s == 0) out += d;
+    else {
+        if ((int)d.size() <= s) d = std::string((size_t)(s + 1 - (int)d.size()), '0') + d;
+        out += d.substr(0, d.size() - (size_t)s) + "." + d.substr(d.size() - (size_t)s);
+    }
+    if (out.size() + 1 > len) return fail(UP_E_NOMEM, "buffer too small (%zu needed)", out.size() + 1);
+    memcpy(buf, out.c_str(), out.size() + 1);
+    return UP_OK;
+}
+
+// ---- diagnostics (no GPU needed): generated source and an NVRTC-only compile
+up_status up_gen_source(const char *variant, const char *expr, const up_column *cols, int ncols, int64_t n_global,
+                        char *buf, size_t len) {
+    if (!variant || !buf) return fail(UP_E_INVAL, "null argument");
+    Typed t;
+    if (up_status s = type_expr(expr, cols, ncols, t)) return s;
+    GenOpts o;
+    o.sum = strcmp(variant, "sum") == 0;
+    const long long N = n_global > 0 ? n_global : (ncols ? cols[0].n : 0);
+    o.LA = o.sum ? limbs_for_precision(sum_precision(t.root->p, N)) : 0;
+    GenInfo info;
+    std::string src = gen_expr_kernel(t.root.get(), t.types, o, info);
+    if (src.size() + 1 > len) return fail(UP_E_NOMEM, "need %zu bytes", src.size() + 1);
+    memcpy(buf, src.c_str(), src.size() + 1);
+    return UP_OK;
+}
+
+up_status up_nvrtc_compile(const char *src, const char *cubin_path, char *log, size_t len) {
+    nvrtcProgram prog;
+    const char *hdrs[2] = {k_up_dev_src, k_up_kparams_src};
+    const char *names[2] = {"up_dev.cuh", "up_kparams.h"};
+    if (nvrtcCreateProgram(&prog, src, "upk.cu", 2, hdrs, names) != NVRTC_SUCCESS)
+        return fail(UP_E_NVRTC, "nvrtcCreateProgram failed");
+    std::vector<const char *> opts(kNvrtcOpts, kNvrtcOpts + sizeof kNvrtcOpts / sizeof kNvrtcOpts[0]);
+    opts.push_back("-Xptxas=-v");
+    nvrtcResult r = nvrtcCompileProgram(prog, (int)opts.size(), opts.data());
+    size_t ls = 0;
+    nvrtcGetProgramLogSize(prog, &ls);
+    std::string lg(ls, '\0');
+    nvrtcGetProgramLog(prog, &lg[0]);
+    if (log && len) { size_t k = std::min(len - 1, lg.size()); memcpy(log, lg.data(), k); log[k] = 0; }
+    if (r != NVRTC_SUCCESS) { nvrtcDestroyProgram(&prog); return fail(UP_E_NVRTC, "NVRTC: %s", nvrtcGetErrorString(r)); }
+    if (cubin_path) {
+        size_t cs = 0;
+        nvrtcGetCUBINSize(prog, &cs);
+        std::vector<char> cubin(cs);
+        nvrtcGetCUBIN(prog, cubin.data());
+        std::ofstream(cubin_path, std::ios::binary).write(cubin.data(), (std::streamsize)cs);
+    }
+    nvrtcDestroyProgram(&prog);
+    return UP_OK;
+}
+
+// modexp / sin_taylor live in special.cpp
+}  // extern "C"
+
+// exported to special.cpp
+up_status up_internal_compile(up_ctx *c, const std::string &src, int rows_per_thread, int ws_slots, int threads,
+                              void **fn_out, int *blocks_per_sm) {
+    JitKernel *k = nullptr;
+    up_status s = compile(c, src, &k);
+    if (s) return s;
+    k->rows_per_thread = rows_per_thread;
+    k->ws_slots = ws_slots;
+    if (threads != k->threads) {
+        k->threads = threads;
+        int nb = 0;
+        CU_TRY(drv.OccupancyMaxActiveBlocksPerMultiprocessor(&nb, k->fn, threads, 0));
+        k->blocks_per_sm = std::max(1, nb);
+    }
+    *fn_out = k;
+    if (blocks_per_sm) *blocks_per_sm = k->blocks_per_sm;
+    return UP_OK;
+}
+up_status up_internal_launch(up_ctx *c, void *kp, up_kparams &P, long long work_items, cudaStream_t st) {
+    return launch(c, (JitKernel *)kp, P, work_items, st);
+}
+std::mutex &up_internal_mutex(up_ctx *c) { return c->mu; }
+unsigned long long *up_internal_ws(up_ctx *c) { return c->d_ws; }
+uint32_t *up_internal_ticket(up_ctx *c) { return c->d_ticket; }
+uint32_t *up_internal_flags(up_ctx *c) { return c->d_flags; }
+up_status up_internal_fail(up_status st, const std::string &msg) { return fail(st, "%s", msg.c_str()); }

@@ -1,0 +1,357 @@
+"""Thin Python binding of libup.so (include/up.h): argument marshalling only.
+
+Every step of the hot path runs in libup's CUDA kernels; PyTorch supplies
+device memory, streams and process groups.  There is no CPU fallback: if the
+extension is missing, importing/using this module raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+from typing import List, Optional, Sequence
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libup.so")
+
+STATUS = {0: "OK", 1: "INVAL", 2: "RANGE", 3: "OVERFLOW", 4: "DIVZERO", 5: "NOMEM",
+          6: "CUDA", 7: "NVRTC", 8: "UNSUPPORTED"}
+
+
+class UpError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"libup {STATUS.get(code, code)}: {msg}")
+        self.code = code
+        self.name = STATUS.get(code, str(code))
+
+
+class up_column(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("ld", ctypes.c_int64), ("p", ctypes.c_int32),
+                ("s", ctypes.c_int32), ("limbs", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("data", ctypes.c_void_p)]
+
+
+_lib = None
+EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_ld", "up_sum_precision",
+           "up_column_from_host_bin", "up_column_from_device_bin", "up_column_from_host",
+           "up_column_to_host_bin", "up_expr_type", "up_eval_expr", "up_sum_type", "up_sum_expr",
+           "up_sum", "up_sum_combine", "up_modexp", "up_modexp_sum_type", "up_modexp_sum",
+           "up_sin_taylor", "up_sin_taylor_sum", "up_check", "up_format_decimal", "up_launch_count",
+           "up_jit_ms", "up_gen_source", "up_nvrtc_compile"]
+
+
+def lib():
+    """Load libup.so (raises if it has not been built: no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} missing: run `python -m paper_conf_icde_lixylz24_b200.build`")
+    L = ctypes.CDLL(LIB_PATH)
+    c = ctypes
+    P = c.c_void_p
+    PC = c.POINTER(up_column)
+    L.up_last_error.restype = c.c_char_p
+    L.up_limbs.argtypes = [c.c_int32]; L.up_limbs.restype = c.c_int32
+    L.up_ld.argtypes = [c.c_int64]; L.up_ld.restype = c.c_int64
+    L.up_sum_precision.argtypes = [c.c_int32, c.c_int64]; L.up_sum_precision.restype = c.c_int32
+    L.up_ctx_create.argtypes = [c.c_int, c.POINTER(P)]
+    L.up_ctx_destroy.argtypes = [P]
+    L.up_column_from_host_bin.argtypes = [P, P, c.c_int32, P, PC, P]
+    L.up_column_from_device_bin.argtypes = [P, P, c.c_int32, P, PC, P]
+    L.up_column_from_host.argtypes = [P, c.POINTER(c.c_char_p), PC, P]
+    L.up_column_to_host_bin.argtypes = [P, PC, P, P, P]
+    L.up_expr_type.argtypes = [P, c.c_char_p, PC, c.c_int, c.POINTER(c.c_int32), c.POINTER(c.c_int32)]
+    L.up_eval_expr.argtypes = [P, c.c_char_p, PC, c.c_int, PC, P]
+    L.up_sum_type.argtypes = [P, c.c_char_p, PC, c.c_int, c.c_int64, c.POINTER(c.c_int32),
+                              c.POINTER(c.c_int32), c.POINTER(c.c_int32)]
+    L.up_sum_expr.argtypes = [P, c.c_char_p, PC, c.c_int, c.c_int64, P, P]
+    L.up_sum.argtypes = [P, PC, c.c_int64, P, P]
+    L.up_sum_combine.argtypes = [P, P, c.c_int32, c.c_int32, P, P]
+    L.up_modexp.argtypes = [P, PC, c.c_char_p, c.c_char_p, PC, P]
+    L.up_modexp_sum_type.argtypes = [P, c.c_char_p, c.c_int64, c.POINTER(c.c_int32), c.POINTER(c.c_int32)]
+    L.up_modexp_sum.argtypes = [P, PC, c.c_char_p, c.c_char_p, c.c_int64, P, P]
+    L.up_sin_taylor.argtypes = [P, PC, c.c_int32, PC, P]
+    L.up_sin_taylor_sum.argtypes = [P, PC, c.c_int32, c.c_int64, P, P]
+    L.up_check.argtypes = [P, P]
+    L.up_format_decimal.argtypes = [P, c.c_int32, c.c_int32, c.c_char_p, c.c_size_t]
+    L.up_launch_count.argtypes = [P]; L.up_launch_count.restype = c.c_uint64
+    L.up_jit_ms.argtypes = [P]; L.up_jit_ms.restype = c.c_double
+    L.up_gen_source.argtypes = [c.c_char_p, c.c_char_p, PC, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
+    L.up_nvrtc_compile.argtypes = [c.c_char_p, c.c_char_p, c.c_char_p, c.c_size_t]
+    _lib = L
+    return L
+
+
+def _chk(code: int):
+    if code != 0:
+        raise UpError(code, lib().up_last_error().decode(errors="replace"))
+
+
+def limbs(p: int) -> int:
+    return lib().up_limbs(p)
+
+
+def ld_for(n: int) -> int:
+    return lib().up_ld(n)
+
+
+def sum_precision(p: int, n_global: int) -> int:
+    return lib().up_sum_precision(p, n_global)
+
+
+def _stream_ptr(stream) -> Optional[int]:
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+class Column:
+    """A DECIMAL(p,s) column on the GPU: `limbs` two's-complement limb planes
+    held in a torch int32 tensor of shape (limbs, ld)."""
+
+    def __init__(self, p: int, s: int, n: int, device="cuda", data=None):
+        import torch
+        self.p, self.s, self.n = p, s, n
+        self.limbs = limbs(p)
+        self.ld = ld_for(n)
+        if data is None:
+            data = torch.empty((self.limbs, max(self.ld, 4)), dtype=torch.int32, device=device)
+        self.data = data
+
+    def desc(self) -> up_column:
+        return up_column(self.n, self.ld, self.p, self.s, self.limbs, 0, self.data.data_ptr())
+
+    @property
+    def type(self):
+        return (self.p, self.s)
+
+
+def _descs(cols: Sequence[Column]):
+    arr = (up_column * max(1, len(cols)))()
+    for i, c in enumerate(cols):
+        arr[i] = c.desc()
+    return arr
+
+
+def format_decimal(limbs_u32: Sequence[int], s: int) -> str:
+    """Canonical string of a two's-complement limb vector (libup's formatter)."""
+    n = len(limbs_u32)
+    arr = (ctypes.c_uint32 * n)(*[int(x) & 0xFFFFFFFF for x in limbs_u32])
+    buf = ctypes.create_string_buffer(n * 10 + s + 8)
+    _chk(lib().up_format_decimal(arr, n, s, buf, len(buf)))
+    return buf.value.decode()
+
+
+def limbs_to_int(limbs_u32: Sequence[int]) -> int:
+    v = 0
+    for x in reversed(list(limbs_u32)):
+        v = (v << 32) | (int(x) & 0xFFFFFFFF)
+    n = len(limbs_u32)
+    if n and (int(limbs_u32[-1]) & 0x80000000):
+        v -= 1 << (32 * n)
+    return v
+
+
+class Context:
+    """One libup context (kernel cache, SUM workspace, staging) on one device."""
+
+    def __init__(self, device: int = 0):
+        import torch
+        torch.cuda.init()
+        torch.cuda.set_device(device)
+        self.device = device
+        h = ctypes.c_void_p()
+        _chk(lib().up_ctx_create(device, ctypes.byref(h)))
+        self.h = h
+
+    def close(self):
+        if self.h:
+            lib().up_ctx_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ------------------------------------------------------------------ info
+    @property
+    def launches(self) -> int:
+        return lib().up_launch_count(self.h)
+
+    @property
+    def jit_ms(self) -> float:
+        return lib().up_jit_ms(self.h)
+
+    # ------------------------------------------------------------------ columns
+    def column_from_host_bin(self, p: int, s: int, mag, neg=None, stream=None, out: Optional[Column] = None):
+        """mag: (n, W) uint32 host array (numpy or pinned torch); neg: (n,) uint8."""
+        import numpy as np
+        import torch
+        if isinstance(mag, np.ndarray):
+            n, W = mag.shape
+            mag_ptr = mag.ctypes.data
+            neg_ptr = neg.ctypes.data if neg is not None else None
+        else:
+            n, W = mag.shape
+            mag_ptr = mag.data_ptr()
+            neg_ptr = neg.data_ptr() if neg is not None else None
+        col = out if out is not None else Column(p, s, n)
+        d = col.desc()
+        _chk(lib().up_column_from_host_bin(self.h, mag_ptr, W, neg_ptr, ctypes.byref(d), _stream_ptr(stream)))
+        return col
+
+    def column_from_device_bin(self, p: int, s: int, d_mag, d_neg=None, stream=None, out: Optional[Column] = None):
+        """d_mag: (n, W) int32/uint32 CUDA tensor; d_neg: (n,) uint8 CUDA tensor."""
+        n, W = d_mag.shape
+        col = out if out is not None else Column(p, s, n)
+        d = col.desc()
+        _chk(lib().up_column_from_device_bin(self.h, d_mag.data_ptr(), W,
+                                             d_neg.data_ptr() if d_neg is not None else None,
+                                             ctypes.byref(d), _stream_ptr(stream)))
+        return col
+
+    def column_from_strings(self, p: int, s: int, values: Sequence[str], stream=None):
+        col = Column(p, s, len(values))
+        arr = (ctypes.c_char_p * max(1, len(values)))(*[v.encode() for v in values])
+        d = col.desc()
+        _chk(lib().up_column_from_host(self.h, arr, ctypes.byref(d), _stream_ptr(stream)))
+        return col
+
+    def column_to_ints(self, col: Column, stream=None) -> List[int]:
+        import numpy as np
+        mag = np.zeros((max(col.n, 1), col.limbs), dtype=np.uint32)
+        neg = np.zeros(max(col.n, 1), dtype=np.uint8)
+        d = col.desc()
+        _chk(lib().up_column_to_host_bin(self.h, ctypes.byref(d), mag.ctypes.data, neg.ctypes.data,
+                                         _stream_ptr(stream)))
+        out = []
+        for i in range(col.n):
+            v = 0
+            for x in reversed(mag[i].tolist()):
+                v = (v << 32) | x
+            out.append(-v if neg[i] else v)
+        return out
+
+    def column_to_strings(self, col: Column, stream=None) -> List[str]:
+        return [_fmt(v, col.s) for v in self.column_to_ints(col, stream)]
+
+    # ------------------------------------------------------------------ expressions
+    def expr_type(self, expr: str, cols: Sequence[Column]):
+        P, S = ctypes.c_int32(), ctypes.c_int32()
+        _chk(lib().up_expr_type(self.h, expr.encode(), _descs(cols), len(cols), ctypes.byref(P), ctypes.byref(S)))
+        return P.value, S.value
+
+    def eval_expr(self, expr: str, cols: Sequence[Column], out: Optional[Column] = None, stream=None) -> Column:
+        p, s = self.expr_type(expr, cols)
+        if out is None:
+            out = Column(p, s, cols[0].n)
+        d = out.desc()
+        _chk(lib().up_eval_expr(self.h, expr.encode(), _descs(cols), len(cols), ctypes.byref(d), _stream_ptr(stream)))
+        return out
+
+    def sum_type(self, expr: str, cols: Sequence[Column], n_global: int = 0):
+        P, S, LA = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+        _chk(lib().up_sum_type(self.h, expr.encode(), _descs(cols), len(cols), n_global,
+                               ctypes.byref(P), ctypes.byref(S), ctypes.byref(LA)))
+        return P.value, S.value, LA.value
+
+    def sum_expr(self, expr: str, cols: Sequence[Column], n_global: int = 0, out=None, stream=None):
+        """SELECT SUM(expr): returns the device tensor of LA two's-complement limbs."""
+        import torch
+        _, _, LA = self.sum_type(expr, cols, n_global)
+        if out is None:
+            out = torch.empty(LA, dtype=torch.int32, device=cols[0].data.device)
+        _chk(lib().up_sum_expr(self.h, expr.encode(), _descs(cols), len(cols), n_global, out.data_ptr(),
+                               _stream_ptr(stream)))
+        return out
+
+    def sum_combine(self, partials, la: int, out=None, stream=None):
+        """partials: (nranks * la) int32 CUDA tensor (e.g. an all-gather output)."""
+        import torch
+        nranks = partials.numel() // la
+        if out is None:
+            out = torch.empty(la, dtype=torch.int32, device=partials.device)
+        _chk(lib().up_sum_combine(self.h, partials.data_ptr(), nranks, la, out.data_ptr(), _stream_ptr(stream)))
+        return out
+
+    def modexp(self, base: Column, exponent: int, modulus: int, out: Optional[Column] = None, stream=None):
+        if out is None:
+            out = Column(len(str(modulus)), 0, base.n)
+        d = out.desc()
+        bd = base.desc()
+        _chk(lib().up_modexp(self.h, ctypes.byref(bd), str(exponent).encode(), str(modulus).encode(),
+                             ctypes.byref(d), _stream_ptr(stream)))
+        return out
+
+    def modexp_sum_type(self, modulus: int, n_global: int):
+        P, LA = ctypes.c_int32(), ctypes.c_int32()
+        _chk(lib().up_modexp_sum_type(self.h, str(modulus).encode(), n_global, ctypes.byref(P), ctypes.byref(LA)))
+        return P.value, LA.value
+
+    def modexp_sum(self, base: Column, exponent: int, modulus: int, n_global: int = 0, out=None, stream=None):
+        import torch
+        _, LA = self.modexp_sum_type(modulus, n_global or base.n)
+        if out is None:
+            out = torch.empty(LA, dtype=torch.int32, device=base.data.device)
+        bd = base.desc()
+        _chk(lib().up_modexp_sum(self.h, ctypes.byref(bd), str(exponent).encode(), str(modulus).encode(),
+                                 n_global, out.data_ptr(), _stream_ptr(stream)))
+        return out
+
+    def sin_taylor(self, x: Column, P: int, out: Optional[Column] = None, stream=None):
+        if out is None:
+            out = Column(P + 1, P, x.n)
+        d, xd = out.desc(), x.desc()
+        _chk(lib().up_sin_taylor(self.h, ctypes.byref(xd), P, ctypes.byref(d), _stream_ptr(stream)))
+        return out
+
+    def sin_taylor_sum(self, x: Column, P: int, n_global: int = 0, out=None, stream=None):
+        import torch
+        LA = limbs(sum_precision(P + 1, n_global or x.n))
+        if out is None:
+            out = torch.empty(LA, dtype=torch.int32, device=x.data.device)
+        xd = x.desc()
+        _chk(lib().up_sin_taylor_sum(self.h, ctypes.byref(xd), P, n_global, out.data_ptr(), _stream_ptr(stream)))
+        return out
+
+    def check(self, stream=None):
+        _chk(lib().up_check(self.h, _stream_ptr(stream)))
+
+
+def _fmt(v: int, s: int) -> str:
+    sign = "-" if v < 0 else ""
+    a = str(abs(v))
+    if s == 0:
+        return sign + a
+    a = a.rjust(s + 1, "0")
+    return sign + a[:-s] + "." + a[-s:]
+
+
+def result_to_string(limb_tensor, s: int) -> str:
+    """Device/host limb tensor of a SUM result -> canonical decimal string."""
+    vals = limb_tensor.detach().cpu().tolist() if hasattr(limb_tensor, "detach") else list(limb_tensor)
+    return format_decimal(vals, s)
+
+
+# ---------------------------------------------------------------------- diagnostics
+def gen_source(variant: str, expr: str, types: Sequence[tuple], n_global: int = 1) -> str:
+    arr = (up_column * max(1, len(types)))()
+    for i, (p, s) in enumerate(types):
+        arr[i] = up_column(n_global, ld_for(n_global), p, s, limbs(p), 0, None)
+    buf = ctypes.create_string_buffer(1 << 24)
+    _chk(lib().up_gen_source(variant.encode(), expr.encode(), arr, len(types), n_global, buf, len(buf)))
+    return buf.value.decode()
+
+
+def nvrtc_compile(src: str, cubin_path: Optional[str] = None) -> str:
+    log = ctypes.create_string_buffer(1 << 16)
+    code = lib().up_nvrtc_compile(src.encode(), cubin_path.encode() if cubin_path else None, log, len(log))
+    if code:
+        raise UpError(code, lib().up_last_error().decode() + "\n" + log.value.decode(errors="replace"))
+    return log.value.decode(errors="replace")

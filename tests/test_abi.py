@@ -1,0 +1,97 @@
+"""Host-side checks of the C-ABI library (no GPU): it loads, exports every
+symbol include/up.h declares, sizes limbs as the paper's table says, formats
+results canonically, and its specialiser emits CUDA that NVRTC compiles for
+sm_100a (register/spill report checked for the hot narrow kernels)."""
+import os
+import random
+import re
+
+import pytest
+
+from paper_conf_icde_lixylz24_b200 import up
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "up.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(up_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_library_loads_and_exports_every_declared_symbol():
+    L = up.lib()
+    names = header_functions()
+    assert len(names) >= 25
+    for n in names:
+        assert hasattr(L, n), n
+    assert set(names) <= set(up.EXPORTS)
+
+
+def test_limb_table_matches_paper():
+    """result precisions 18/38/76/153/307 <-> LEN 2/4/8/16/32
+    (reading Q1: exact for the sign-bit rule 10^p <= 2^(32L-1))."""
+    for p, L in [(18, 2), (38, 4), (76, 8), (153, 16), (307, 32)]:
+        assert up.limbs(p) == L
+        assert up.limbs(p + 1) == L + 1
+    for p in range(1, 400):
+        L = up.limbs(p)
+        assert 10 ** p <= 2 ** (32 * L - 1) and (L == 1 or 10 ** p > 2 ** (32 * (L - 1) - 1))
+
+
+def test_sum_precision_rule():
+    assert up.sum_precision(18, 1_000_000) == 24
+    assert up.sum_precision(36, 10_000_000) == 43
+    assert up.sum_precision(36, 10_000_001) == 44
+    assert up.sum_precision(36, 1) == 36
+    assert up.ld_for(5) == 8 and up.ld_for(8) == 8 and up.ld_for(0) == 0
+
+
+def test_format_decimal_canonical():
+    rng = random.Random(3)
+    for _ in range(200):
+        n = rng.randint(1, 6)
+        v = rng.randrange(-(2 ** (32 * n - 1)), 2 ** (32 * n - 1))
+        s = rng.randint(0, 30)
+        limbs = [(v >> (32 * j)) & 0xFFFFFFFF for j in range(n)]
+        want = ("-" if v < 0 else "") + (lambda a: a if s == 0 else a[:-s] + "." + a[-s:])(str(abs(v)).rjust(s + 1, "0"))
+        assert up.format_decimal(limbs, s) == want
+    assert up.format_decimal([0, 0], 3) == "0.000"
+
+
+def test_expression_typing_on_host():
+    """up_expr_type runs on the host (no GPU): the paper's rules."""
+    src = up.gen_source("eval", "c1*c2 - c3/c4", [(200, 50)] * 4, 100)
+    assert "type (401,100)" in src
+    assert "type (18,5) L=2" in up.gen_source("sum", "c1+c2", [(17, 5), (14, 2)], 10)
+    assert "type (36,5) L=4" in up.gen_source("sum", "c1+c2", [(35, 5), (32, 2)], 10)
+    with pytest.raises(up.UpError) as ei:
+        up.gen_source("eval", "c1 % c2", [(10, 2), (10, 0)], 10)
+    assert ei.value.name == "INVAL"
+    with pytest.raises(up.UpError):
+        up.gen_source("eval", "c1 + c3", [(10, 2), (10, 0)], 10)
+    with pytest.raises(up.UpError):
+        up.gen_source("eval", "c1 + ", [(10, 2)], 10)
+
+
+def _regs(log):
+    m = re.search(r"Used (\d+) registers", log)
+    sp = re.search(r"(\d+) bytes spill stores", log)
+    return int(m.group(1)), int(sp.group(1)) if sp else 0
+
+
+@pytest.mark.parametrize("variant,expr,types", [
+    ("sum", "c1+c2", [(17, 5), (14, 2)]),
+    ("sum", "c1+c2", [(35, 5), (32, 2)]),
+    ("eval", "c1+c2", [(35, 5), (32, 2)]),
+    ("sum", "c1*c2 - c3/c4", [(30, 10)] * 4),
+    ("eval", "c1 % c2 * c1 % c2", [(40, 0), (41, 0)]),
+    ("sum", "-c1/(c2+0.5)", [(12, 3), (9, 2)]),
+])
+def test_specialised_kernels_compile_for_sm100a(variant, expr, types, tmp_path):
+    src = up.gen_source(variant, expr, types, 1_000_000)
+    log = up.nvrtc_compile(src, str(tmp_path / "k.cubin"))
+    regs, spills = _regs(log)
+    assert (tmp_path / "k.cubin").stat().st_size > 0
+    if expr == "c1+c2":
+        assert spills == 0 and regs <= 64, log
