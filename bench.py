@@ -1,23 +1,24 @@
 #!/usr/bin/env python
-"""bench.py -- tuples/s for SELECT SUM(expr) over DECIMAL columns on B200.
+"""bench.py -- tuples/s for SELECT SUM(...) over DECIMAL columns on B200.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C] [--impl up|reference]
 
 Default workload = BASELINE.json configs[1] (the paper's Fig. 1 high-p query):
 SELECT SUM(c1+c2), 10M tuples per GPU, c1 DECIMAL(35,5), c2 DECIMAL(32,2).
-A step = one pass of the whole hot path over the resident columns:
-fused eval+SUM kernel (+ NCCL all-gather of the partials and the exact
-combine kernel when N > 1).  Inputs are seeded synthetic columns (gen/),
-larger than L2 (no flush needed).  For N > 1 rows are sharded (weak
-scaling: every rank owns `rows` rows; typing uses the global row count).
-
-Also reported: `e2e` (same metric through the C ABI from pinned HOST buffers,
-H2D + ingestion + SUM + D2H of the result inside the timed region),
-`roofline` (fused kernel's algorithmic bytes / kernel time vs the measured
-HBM copy bandwidth), `cpu_baseline` (the CPU oracle, as it stands, timed on
-the host cores on a bounded sample), clocks sampled with NVML during the
-timed region, and `gpu_launches` (libup kernels launched in the timed region).
-`--impl reference` times the CPU oracle instead (the reference arm).
+Other configs (parity-test cases by default, bench lines on request):
+  1  SUM(c1+c2) DECIMAL(17,5)+DECIMAL(14,2), 1M tuples (L2-resident: flushed)
+  3  SUM(c1*c2 - c3/c4) DECIMAL(200,50) x4, 12.5M tuples/GPU (100M on 8)
+  4  SUM(x^65537 mod N), 1024-bit N, 10M tuples (RSA, Query 4 generalised)
+  5  SUM(sin_P(x)), P = 1000 digits, x ~ N(0.78, 0.01) DECIMAL(9,8), 1M tuples
+A step = one pass of the whole hot path over the resident columns: the fused
+kernel (+ NCCL all-gather of the partials and the exact combine kernel when
+N > 1).  Inputs are seeded synthetic columns (gen/).  For N > 1 rows are
+sharded (weak scaling: every rank owns `rows` rows; typing uses the global
+row count).  Reported with it: `e2e` (same metric through the C ABI from
+pinned HOST buffers: H2D + ingestion + SUM + D2H of the result in the timed
+region), `roofline` of the fused kernel, `cpu_baseline` (the CPU oracle as it
+stands on a bounded sample), NVML clocks during the timed region, and
+`gpu_launches`.  `--impl reference` times the CPU oracle (the reference arm).
 """
 from __future__ import annotations
 
@@ -32,14 +33,20 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "tuples/sec for SELECT SUM(expr) by DECIMAL precision at 1/2/4/8 B200; % HBM/INT peak"
+# IMAD-pipe peak: 64 lanes/clk/SM (fma pipe, 2 cycles per warp instruction per
+# SMSP; B300_MICROARCH "Pipe rates") x 148 SMs x 1965 MHz max SM clock.
+IMAD_PEAK_TOPS = 64 * 148 * 1.965e9 / 1e12
 
 CONFIGS = {
-    1: dict(name="cfg1 SUM(c1+c2) DECIMAL(17,5)+DECIMAL(14,2)", expr="c1+c2", types=[(17, 5), (14, 2)],
-            rows=1_000_000, bound="hbm"),
-    2: dict(name="cfg2 SUM(c1+c2) DECIMAL(35,5)+DECIMAL(32,2) (Fig.1 high-p)", expr="c1+c2",
-            types=[(35, 5), (32, 2)], rows=10_000_000, bound="hbm"),
-    3: dict(name="cfg3 SUM(c1*c2 - c3/c4) DECIMAL(200,50)", expr="c1*c2 - c3/c4", types=[(200, 50)] * 4,
-            rows=12_500_000, bound="alu", lead=(3,)),
+    1: dict(kind="expr", name="cfg1 SUM(c1+c2) DECIMAL(17,5)+DECIMAL(14,2)", expr="c1+c2",
+            types=[(17, 5), (14, 2)], rows=1_000_000),
+    2: dict(kind="expr", name="cfg2 SUM(c1+c2) DECIMAL(35,5)+DECIMAL(32,2) (Fig.1 high-p)", expr="c1+c2",
+            types=[(35, 5), (32, 2)], rows=10_000_000),
+    3: dict(kind="expr", name="cfg3 SUM(c1*c2 - c3/c4) DECIMAL(200,50)", expr="c1*c2 - c3/c4",
+            types=[(200, 50)] * 4, rows=12_500_000, lead=(3,)),
+    4: dict(kind="modexp", name="cfg4 SUM(x^65537 mod N) 1024-bit RSA", bits=1024, e=65537, rows=10_000_000),
+    5: dict(kind="sin", name="cfg5 SUM(sin_P(x)) P=1000, x~N(0.78,0.01) DECIMAL(9,8)", P=1000, mu=0.78,
+            rows=1_000_000),
 }
 
 
@@ -107,26 +114,204 @@ def dist_env():
     return ws, rank, local
 
 
-def cpu_baseline(cfg, host_cols, budget_s=12.0):
-    """The oracle (oracle/updec.c, as it stands) on a bounded row sample,
-    all host cores (pthreads, static row blocks, exact combine)."""
-    import oracle
+# --------------------------------------------------------------------------- workloads
+class Workload:
+    """Inputs (device-resident + pinned-host copies) and the step for one config."""
+
+    def __init__(self, cfg, args, ctx, rows, n_global, row0):
+        self.cfg, self.args, self.ctx = cfg, args, ctx
+        self.rows, self.n_global, self.row0 = rows, n_global, row0
+
+
+class ExprWorkload(Workload):
+    def setup(self):
+        from gen import device as gdev
+        from paper_conf_icde_lixylz24_b200 import up
+        cfg, ctx = self.cfg, self.ctx
+        self.raw, self.cols = [], []
+        for k, (p, s) in enumerate(cfg["types"]):
+            mag, neg = gdev.uniform_decimal(self.rows, p, self.args.config, k + 1, row0=self.row0,
+                                            nonzero_lead=(k in cfg.get("lead", ())))
+            self.raw.append((mag, neg))
+            self.cols.append(ctx.column_from_device_bin(p, s, mag, neg))
+        ctx.check()
+        self.P, self.S, self.LA = ctx.sum_type(cfg["expr"], self.cols, self.n_global)
+        self.e2e_cols = [up.Column(p, s, self.rows) for p, s in cfg["types"]]
+        self.bytes_per_row = sum(4 * up.limbs(p) for p, s in cfg["types"])
+
+    def kernel(self, out):
+        self.ctx.sum_expr(self.cfg["expr"], self.cols, self.n_global, out=out)
+
+    def e2e_ingest(self, host):
+        for (hm, hn), (p, s), col in zip(host, self.cfg["types"], self.e2e_cols):
+            self.ctx.column_from_host_bin(p, s, hm, hn, out=col)
+
+    def e2e_kernel(self, out):
+        self.ctx.sum_expr(self.cfg["expr"], self.e2e_cols, self.n_global, out=out)
+
+    def roofline(self, kernel_ms, peaks):
+        if self.cfg["types"][0][0] >= 100:     # wide expressions: integer-pipe bound
+            return self._alu_roofline(kernel_ms, self.alg_imad_per_row())
+        alg = self.bytes_per_row * self.rows
+        peak = peaks.get("hbm_gbs", 6650.0)
+        ach = alg / (kernel_ms / 1e3) / 1e9
+        return {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(ach / peak, 4), "kernel_ms": round(kernel_ms, 5), "alg_bytes_per_launch": alg,
+                "alg_unit": f"{self.bytes_per_row} B/row (limb planes read) x {self.rows} rows",
+                "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks
+                else "fallback 6.65 TB/s"}
+
+    def alg_imad_per_row(self):
+        """limb products of c1*c2 - c3/c4 = x (L*L) + / prescale
+        (L x limbs(10^(s+4))) + / (quotient limbs x L) + alignment of the
+        quotient (limbs(q) x limbs(10^(2s-(s+4)))); 2 IMAD per limb product."""
+        from paper_conf_icde_lixylz24_b200 import up
+        p, s = self.cfg["types"][0]
+        mag = lambda k: max(1, (10 ** k).bit_length() // 32 + 1)   # noqa: E731
+        L = up.limbs(p)
+        nu = mag(p + s + 4)
+        products = L * L + L * mag(s + 4) + (nu - L + 1) * L + up.limbs(s + 5) * mag(s - 4)
+        return 2 * products
+
+    def _alu_roofline(self, kernel_ms, imad_per_row):
+        ops = imad_per_row * self.rows
+        ach = ops / (kernel_ms / 1e3) / 1e12
+        return {"bound": "alu", "achieved": round(ach, 3), "peak": round(IMAD_PEAK_TOPS, 2), "unit": "T IMAD/s",
+                "frac": round(ach / IMAD_PEAK_TOPS, 4), "kernel_ms": round(kernel_ms, 4),
+                "alg_ops_per_launch": ops,
+                "alg_unit": f"{imad_per_row} IMAD-pipe ops/row (2 per 32x32 limb product) x {self.rows} rows",
+                "peak_source": "derived: 64 IMAD lanes/clk/SM x 148 SMs x 1965 MHz (DESIGN.md)"}
+
+    def host_for_oracle(self):
+        import numpy as np
+        import oracle
+        return [oracle.Column(p, s, m.cpu().numpy().view(np.uint32), g.cpu().numpy())
+                for (m, g), (p, s) in zip(self.raw, self.cfg["types"])]
+
+    def oracle_sum(self, ocols, n, threads):
+        import oracle
+        return oracle.eval_sum(self.cfg["expr"], [c.head(n) for c in ocols], n=n, n_global=self.n_global,
+                               threads=threads)[0]
+
+    def workload_desc(self):
+        return {"expr": self.cfg["expr"], "types": self.cfg["types"], "sum_type": [self.P, self.S],
+                "sum_limbs": self.LA}
+
+
+class ModexpWorkload(ExprWorkload):
+    def setup(self):
+        from gen import device as gdev
+        from gen import synth
+        from paper_conf_icde_lixylz24_b200 import up
+        cfg, ctx = self.cfg, self.ctx
+        self.N, _, _ = synth.rsa_modulus(cfg["bits"])
+        self.e = cfg["e"]
+        self.d = len(str(self.N))
+        mag, neg = gdev.uniform_range(synth.SEED, synth.stream_id(4, 0), self.rows, 0, self.N - 1, signed=False,
+                                      row0=self.row0)
+        self.raw = [(mag, neg)]
+        self.cols = [ctx.column_from_device_bin(self.d, 0, mag, neg)]
+        ctx.check()
+        self.P, self.LA = ctx.modexp_sum_type(self.N, self.n_global)
+        self.S = 0
+        self.e2e_cols = [up.Column(self.d, 0, self.rows)]
+        self.cfg = dict(cfg, types=[(self.d, 0)])
+
+    def kernel(self, out):
+        self.ctx.modexp_sum(self.cols[0], self.e, self.N, self.n_global, out=out)
+
+    def e2e_kernel(self, out):
+        self.ctx.modexp_sum(self.e2e_cols[0], self.e, self.N, self.n_global, out=out)
+
+    def roofline(self, kernel_ms, peaks):
+        n = (self.N.bit_length() + 31) // 32
+        montmuls = (self.e.bit_length() - 1) + bin(self.e).count("1") - 1 + 2   # squarings + multiplies + in/out
+        return self._alu_roofline(kernel_ms, 2 * montmuls * (2 * n * n + n))
+
+    def oracle_sum(self, ocols, n, threads):
+        import oracle
+        return oracle.modexp_sum(ocols[0].head(n), self.e, self.N, threads=threads)
+
+    def workload_desc(self):
+        return {"modulus_bits": self.N.bit_length(), "e": self.e, "base_type": [self.d, 0],
+                "sum_type": [self.P, 0], "sum_limbs": self.LA}
+
+
+class SinWorkload(ExprWorkload):
+    def setup(self):
+        import torch
+        from gen import synth
+        from paper_conf_icde_lixylz24_b200 import up
+        cfg, ctx = self.cfg, self.ctx
+        self.Pd = cfg["P"]
+        mag, neg = synth.normal_decimal(self.rows, cfg["mu"], 0.01, 8, config=5, column=0, row0=self.row0)
+        self.host_np = (mag, neg)
+        tm = torch.from_numpy(mag.view("int32")).cuda()
+        tn = torch.from_numpy(neg).cuda()
+        self.raw = [(tm, tn)]
+        self.cols = [ctx.column_from_device_bin(9, 8, tm, tn)]
+        ctx.check()
+        self.P = up.sum_precision(self.Pd + 1, self.n_global)
+        self.S = self.Pd
+        self.LA = up.limbs(self.P)
+        self.e2e_cols = [up.Column(9, 8, self.rows)]
+        self.cfg = dict(cfg, types=[(9, 8)])
+        # mean number of Taylor terms (for the algorithmic op count), from a sample
+        import numpy as np
+        ks = []
+        for m in mag[: 256, 0].tolist():
+            t, k = m * 10 ** (self.Pd - 8), 1
+            while t:
+                t = t * m * m // (10 ** 16 * (2 * k) * (2 * k + 1))
+                k += 1
+            ks.append(k - 1)
+        self.mean_terms = float(np.mean(ks))
+
+    def kernel(self, out):
+        self.ctx.sin_taylor_sum(self.cols[0], self.Pd, self.n_global, out=out)
+
+    def e2e_kernel(self, out):
+        self.ctx.sin_taylor_sum(self.e2e_cols[0], self.Pd, self.n_global, out=out)
+
+    def roofline(self, kernel_ms, peaks):
+        from paper_conf_icde_lixylz24_b200 import up
+        W = up.limbs(self.Pd + 23)
+        # per term and limb: x m_x^2 (2 limb products = 4 IMAD) + 3 short-division
+        # steps (64x64 high product ~4 IMAD + q*d 1 IMAD each) = 19 IMAD-pipe ops
+        per_row = int(self.mean_terms * W * 19)
+        r = self._alu_roofline(kernel_ms, per_row)
+        r["alg_unit"] += f"; mean {self.mean_terms:.1f} terms x {W} limbs x 19"
+        return r
+
+    def oracle_sum(self, ocols, n, threads):
+        import oracle
+        return oracle.sin_sum(ocols[0].head(n), self.Pd, threads=threads)
+
+    def workload_desc(self):
+        return {"P": self.Pd, "x_type": [9, 8], "mu": self.cfg["mu"], "sigma": 0.01, "sum_type": [self.P, self.S],
+                "sum_limbs": self.LA}
+
+
+KINDS = {"expr": ExprWorkload, "modexp": ModexpWorkload, "sin": SinWorkload}
+
+
+def cpu_baseline(wl, budget_s=12.0):
+    """The oracle (oracle/updec.c, as it stands) on a bounded row sample, all
+    host cores (pthreads, static row blocks, exact combine)."""
     cores = len(os.sched_getaffinity(0))
-    ocols = [oracle.Column(p, s, m, g) for (m, g), (p, s) in zip(host_cols, cfg["types"])]
-    n_all = host_cols[0][0].shape[0]
-    n = min(n_all, 20000)
+    ocols = wl.host_for_oracle()
+    n_all = ocols[0].n
+    n = min(n_all, 64)
     t0 = time.perf_counter()
-    oracle.eval_sum(cfg["expr"], [c.head(n) for c in ocols], n=n, n_global=n_all, threads=cores)
+    wl.oracle_sum(ocols, n, cores)
     dt = time.perf_counter() - t0
-    # scale the sample to ~budget_s of CPU work (bounded by the rows we have)
-    n2 = int(min(n_all, max(n, n * budget_s / max(dt, 1e-3) * 0.8)))
-    if n2 > n:
+    while dt < budget_s / 8 and n < n_all:
+        n = int(min(n_all, n * max(2.0, budget_s / 2 / max(dt, 1e-4))))
         t0 = time.perf_counter()
-        oracle.eval_sum(cfg["expr"], [c.head(n2) for c in ocols], n=n2, n_global=n_all, threads=cores)
+        wl.oracle_sum(ocols, n, cores)
         dt = time.perf_counter() - t0
-        n = n2
     return {"value": n / dt, "unit": "tuples/s", "cores": cores, "kind": "oracle",
-            "sample": f"first {n} of {n_all} rows of the same seeded workload, SUM({cfg['expr']}), "
+            "sample": f"first {n} of {n_all} rows of the same seeded workload ({wl.cfg['name']}), "
                       f"{cores} threads, {dt:.2f} s"}
 
 
@@ -135,20 +320,33 @@ def run_reference(args, cfg):
     ws, rank, _ = dist_env()
     if rank != 0:
         return 0
+    import numpy as np
     import oracle
     from gen import synth
     cores = len(os.sched_getaffinity(0))
     rows = args.rows or cfg["rows"]
     sample = min(rows, args.ref_rows)
-    host = []
-    for k, (p, s) in enumerate(cfg["types"]):
-        host.append(synth.uniform_decimal(sample, p, args.config, k + 1, nonzero_lead=(k in cfg.get("lead", ()))))
-    ocols = [oracle.Column(p, s, m, g) for (m, g), (p, s) in zip(host, cfg["types"])]
+    if cfg["kind"] == "expr":
+        host = [synth.uniform_decimal(sample, p, args.config, k + 1, nonzero_lead=(k in cfg.get("lead", ())))
+                for k, (p, s) in enumerate(cfg["types"])]
+        ocols = [oracle.Column(p, s, m, g) for (m, g), (p, s) in zip(host, cfg["types"])]
+        fn = lambda: oracle.eval_sum(cfg["expr"], ocols, n_global=rows * ws, threads=cores)  # noqa: E731
+    elif cfg["kind"] == "modexp":
+        N, _, _ = synth.rsa_modulus(cfg["bits"])
+        sample = min(sample, 2000)
+        m, g = synth.rsa_messages(sample, N)
+        col = oracle.Column(len(str(N)), 0, m, g)
+        fn = lambda: oracle.modexp_sum(col, cfg["e"], N, threads=cores)  # noqa: E731
+    else:
+        sample = min(sample, 2000)
+        m, g = synth.normal_decimal(sample, cfg["mu"], 0.01, 8, config=5, column=0)
+        col = oracle.Column(9, 8, m, g)
+        fn = lambda: oracle.sin_sum(col, cfg["P"], threads=cores)  # noqa: E731
     for _ in range(args.warmup):
-        oracle.eval_sum(cfg["expr"], ocols, n_global=rows * ws, threads=cores)
+        fn()
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        oracle.eval_sum(cfg["expr"], ocols, n_global=rows * ws, threads=cores)
+        fn()
     dt = (time.perf_counter() - t0) / args.steps
     val = sample / dt
     line = {
@@ -167,25 +365,43 @@ def run_reference(args, cfg):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
-    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=0, help="timed steps (default per config)")
+    ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", type=int, default=2)
     ap.add_argument("--rows", type=int, default=0, help="rows per GPU (default: the config's)")
     ap.add_argument("--impl", default="up", choices=["up", "reference"])
     ap.add_argument("--ref-rows", type=int, default=200_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=0)
+    ap.add_argument("--P", type=int, default=0, help="cfg5 digits")
+    ap.add_argument("--bits", type=int, default=0, help="cfg4 modulus bits")
+    ap.add_argument("--e", type=int, default=0, help="cfg4 exponent")
+    ap.add_argument("--p", type=int, default=0, help="cfg3 precision (scale from the config table)")
     args = ap.parse_args()
-    cfg = CONFIGS[args.config]
+    cfg = dict(CONFIGS[args.config])
+    if args.P:
+        cfg["P"] = args.P
+        cfg["name"] = cfg["name"].replace("P=1000", f"P={args.P}")
+    if args.bits:
+        cfg["bits"] = args.bits
+        cfg["name"] = cfg["name"].replace("1024-bit", f"{args.bits}-bit")
+    if args.e:
+        cfg["e"] = args.e
+        cfg["name"] = cfg["name"].replace("65537", str(args.e))
+    if args.p:
+        s = {200: 50, 500: 75, 1000: 100}.get(args.p, args.p // 4)
+        cfg["types"] = [(args.p, s)] * 4
+        cfg["name"] = f"cfg3 SUM(c1*c2 - c3/c4) DECIMAL({args.p},{s})"
+    if not args.steps:
+        args.steps = {"expr": 200, "modexp": 5, "sin": 3}[cfg["kind"]] if cfg["kind"] != "expr" or \
+            cfg["types"][0][0] < 100 else 5
     if args.impl == "reference":
         return run_reference(args, cfg)
 
-    import numpy as np
     import torch
     import torch.distributed as dist
 
     from gen import device as gdev
-    from gen import synth
     from paper_conf_icde_lixylz24_b200 import up
 
     ws, rank, local = dist_env()
@@ -196,30 +412,25 @@ def main():
     stream = torch.cuda.current_stream()
     rows = args.rows or cfg["rows"]
     n_global = rows * ws
-    row0 = rank * rows
-
-    # ---- inputs: device generator (bit-identical to the host twin), resident in HBM
     gdev.build()
-    cols, raw = [], []
-    for k, (p, s) in enumerate(cfg["types"]):
-        mag, neg = gdev.uniform_decimal(rows, p, args.config, k + 1, row0=row0,
-                                        nonzero_lead=(k in cfg.get("lead", ())))
-        raw.append((mag, neg))
-        cols.append(ctx.column_from_device_bin(p, s, mag, neg))
-    ctx.check()
-    P, S, LA = ctx.sum_type(cfg["expr"], cols, n_global)
+    wl = KINDS[cfg["kind"]](cfg, args, ctx, rows, n_global, rank * rows)
+    wl.setup()
+    LA = wl.LA
     partial = torch.empty(LA, dtype=torch.int32, device="cuda")
     gathered = torch.empty(LA * ws, dtype=torch.int32, device="cuda")
     total = torch.empty(LA, dtype=torch.int32, device="cuda")
+    # L2 flush buffer for working sets below L2 (cfg1: 16 MB)
+    flush = None
+    if getattr(wl, "bytes_per_row", 0) * rows < 256e6 and cfg["kind"] == "expr" and cfg["types"][0][0] < 100:
+        flush = torch.empty(int(256e6) // 4, dtype=torch.int32, device="cuda")
 
     def step():
-        ctx.sum_expr(cfg["expr"], cols, n_global, out=partial)
+        wl.kernel(partial)
         if ws > 1:
             dist.all_gather_into_tensor(gathered, partial)
             ctx.sum_combine(gathered, LA, out=total)
 
-    # warm-up (specialises + JIT-compiles the kernel: excluded from timing)
-    for _ in range(max(3, args.warmup)):
+    for _ in range(max(3, args.warmup)):     # warm-up (includes the one-time specialisation / JIT)
         step()
     ctx.check()
     torch.cuda.synchronize()
@@ -227,26 +438,28 @@ def main():
     # ---- timed region: K steps, barrier + sync on both sides, CUDA events
     K = args.steps
     kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
-    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
     l0 = ctx.launches
     if ws > 1:
         dist.barrier()
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
-        t_start.record(stream)
         for i in range(K):
+            if flush is not None:
+                flush.zero_()            # evict the inputs from L2 (outside the step's events)
+            sev[i][0].record(stream)
             kev[i][0].record(stream)
-            ctx.sum_expr(cfg["expr"], cols, n_global, out=partial)
+            wl.kernel(partial)
             kev[i][1].record(stream)
             if ws > 1:
                 dist.all_gather_into_tensor(gathered, partial)
                 ctx.sum_combine(gathered, LA, out=total)
-        t_end.record(stream)
+            sev[i][1].record(stream)
         torch.cuda.synchronize()
     if ws > 1:
         dist.barrier()
     launches = ctx.launches - l0
-    ms = t_start.elapsed_time(t_end)
+    ms = sum(a.elapsed_time(b) for a, b in sev)
     kernel_ms = sum(a.elapsed_time(b) for a, b in kev) / K
     if ws > 1:
         t = torch.tensor([ms], dtype=torch.float64, device="cuda")
@@ -255,42 +468,31 @@ def main():
     ms_per_step = ms / K
     value = n_global / (ms_per_step / 1e3)
     ctx.check()
-    result = up.result_to_string(total if ws > 1 else partial, S)
-
-    # ---- roofline of the fused kernel (algorithmic bytes: the limb planes read)
-    bytes_per_row = sum(4 * up.limbs(p) for p, s in cfg["types"])
-    alg_bytes = bytes_per_row * rows
+    result = up.result_to_string(total if ws > 1 else partial, wl.S)
     peaks = _peaks()
-    peak = peaks.get("hbm_gbs", 6650.0)
-    achieved = alg_bytes / (kernel_ms / 1e3) / 1e9
-    traffic = None
+    roofline = wl.roofline(kernel_ms, peaks)
     tp = os.path.join(ROOT, "profiles", f"traffic_cfg{args.config}.json")
+    roofline["traffic"] = None
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+            roofline["traffic"] = json.load(open(tp)).get("dram_bytes_per_launch")
         except Exception:
-            traffic = None
-    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "traffic": traffic,
-                "kernel_ms": round(kernel_ms, 5), "alg_bytes_per_launch": alg_bytes,
-                "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s"}
+            pass
 
     # ---- e2e through the C ABI from pinned host buffers
     host = []
-    for mag, neg in raw:
+    for mag, neg in wl.raw:
         hm = torch.empty(mag.shape, dtype=torch.int32, pin_memory=True)
         hn = torch.empty(neg.shape, dtype=torch.uint8, pin_memory=True)
         hm.copy_(mag)
         hn.copy_(neg)
         host.append((hm, hn))
     torch.cuda.synchronize()
-    e2e_cols = [up.Column(p, s, rows) for p, s in cfg["types"]]
     res_host = torch.empty(LA, dtype=torch.int32, pin_memory=True)
 
     def e2e_step():
-        for (hm, hn), (p, s), col in zip(host, cfg["types"], e2e_cols):
-            ctx.column_from_host_bin(p, s, hm, hn, out=col)
-        ctx.sum_expr(cfg["expr"], e2e_cols, n_global, out=partial)
+        wl.e2e_ingest(host)
+        wl.e2e_kernel(partial)
         if ws > 1:
             dist.all_gather_into_tensor(gathered, partial)
             ctx.sum_combine(gathered, LA, out=total)
@@ -298,7 +500,7 @@ def main():
         else:
             res_host.copy_(partial, non_blocking=True)
 
-    for _ in range(3):
+    for _ in range(2):
         e2e_step()
     torch.cuda.synchronize()
     K2 = args.e2e_steps or max(3, min(K, 20))
@@ -317,25 +519,26 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ems = float(t.item())
     ctx.check()
-    assert up.format_decimal(res_host.tolist(), S) == result, "e2e result differs from the device-resident run"
+    assert up.format_decimal(res_host.tolist(), wl.S) == result, "e2e result differs from the resident run"
     h2d = sum(hm.numel() * 4 + hn.numel() for hm, hn in host)
     e2e = {"value": n_global / (ems / K2 / 1e3), "unit": "tuples/s", "h2d_bytes_per_step": h2d,
            "d2h_bytes_per_step": LA * 4, "ms_per_step": ems / K2}
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
-        hc = [(m.cpu().numpy().view(np.uint32), g.cpu().numpy()) for m, g in raw]
-        cpu = cpu_baseline(cfg, hc)
+        cpu = cpu_baseline(wl)
 
     if rank == 0:
+        desc = {"workload": cfg["name"], "rows_per_gpu": rows, "global_rows": n_global,
+                "parallelism": f"rows sharded x{ws}, NCCL all-gather of partials + exact combine" if ws > 1
+                else "1 GPU",
+                "l2": ("flushed before every step (256 MB write)" if flush is not None
+                       else "inputs larger than L2 or compute-bound (no flush)")}
+        desc.update(wl.workload_desc())
         line = {
             "metric": METRIC, "value": value, "unit": "tuples/s", "n_gpus": ws, "steps": K,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": cfg["name"], "expr": cfg["expr"], "types": cfg["types"],
-                       "rows_per_gpu": rows, "global_rows": n_global, "sum_type": [P, S], "sum_limbs": LA,
-                       "parallelism": f"rows sharded x{ws}, NCCL all-gather of partials" if ws > 1 else "1 GPU",
-                       "l2": "inputs %.0f MB/GPU > 126 MB L2 (no flush)" % (alg_bytes / 1e6)},
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic", "config": desc,
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
             "clocks": clk.summary(), "result": result, "jit_ms": round(ctx.jit_ms, 1),
         }

@@ -182,6 +182,14 @@ double up_jit_ms(up_ctx *ctx);
 up_status up_gen_source(const char *variant, const char *expr, const up_column *cols, int ncols,
                         int64_t n_global, char *buf, size_t len);
 up_status up_nvrtc_compile(const char *src, const char *cubin_path, char *log, size_t len);
+/* Compile a generated source into the on-disk cubin cache ($UP_JIT_CACHE,
+ * else <dir of libup.so>/_jitcache) so a GPU process loads it without NVRTC. */
+up_status up_jit_prewarm(const char *src);
+/* Generated sin_taylor source for x DECIMAL(p,s) (sum != 0: fused SUM variant). */
+up_status up_gen_sin_source(int32_t P, int32_t p, int32_t s, int sum, int64_t n_global, char *buf, size_t len);
+/* Generated modexp source for a DECIMAL(base_p,0) base (sum != 0: fused SUM variant). */
+up_status up_gen_modexp_source(const char *exponent, const char *modulus, int32_t base_p, int sum,
+                               int64_t n_global, char *buf, size_t len);
 
 #ifdef __cplusplus
 }

@@ -1,6 +1,9 @@
 // up_host.cpp -- the C ABI of libup.so (include/up.h): context, NVRTC
 // specialisation + kernel cache (row a2), launches, column codec, combine.
 #include <cuda.h>
+#include <dlfcn.h>
+#include <sys/stat.h>
+#include <unistd.h>
 #include <cuda_runtime.h>
 #include <nvrtc.h>
 
@@ -10,6 +13,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <fstream>
+#include <iterator>
 #include <map>
 #include <memory>
 #include <mutex>
@@ -169,14 +173,53 @@ up_status check_column(const up_column *col, const char *what) {
 
 const char *kNvrtcOpts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-default-device", "-lineinfo", "-DNDEBUG"};
 
-up_status compile(up_ctx *c, const std::string &src, JitKernel **out) {
-    auto it = c->by_src.find(src);
-    if (it != c->by_src.end()) { *out = it->second.get(); return UP_OK; }
-    auto t0 = std::chrono::steady_clock::now();
-    if (const char *dump = getenv("UP_DUMP_DIR")) {
-        std::string path = std::string(dump) + "/upk_" + std::to_string(c->by_src.size()) + ".cu";
-        std::ofstream(path) << src;
+// On-disk cubin cache (keyed by FNV-1a of source + options + embedded header):
+// $UP_JIT_CACHE, else <dir of libup.so>/_jitcache.  Purely a compile-time
+// saving; a miss recompiles with NVRTC.
+uint64_t fnv1a(const std::string &s, uint64_t h = 1469598103934665603ull) {
+    for (unsigned char ch : s) { h ^= ch; h *= 1099511628211ull; }
+    return h;
+}
+std::string cache_dir() {
+    if (const char *e = getenv("UP_JIT_CACHE")) return e;
+    Dl_info info;
+    if (dladdr((void *)&fnv1a, &info) && info.dli_fname) {
+        std::string f = info.dli_fname;
+        size_t k = f.rfind('/');
+        if (k != std::string::npos) return f.substr(0, k) + "/_jitcache";
     }
+    return "";
+}
+std::string cache_path(const std::string &src) {
+    std::string d = cache_dir();
+    if (d.empty()) return "";
+    uint64_t h = fnv1a(src);
+    for (const char *o : kNvrtcOpts) h = fnv1a(o, h);
+    h = fnv1a(k_up_dev_src, h);
+    h = fnv1a(k_up_kparams_src, h);
+    char name[64];
+    snprintf(name, sizeof name, "/%016llx.cubin", (unsigned long long)h);
+    return d + name;
+}
+bool read_file(const std::string &path, std::vector<char> &out) {
+    std::ifstream f(path, std::ios::binary);
+    if (!f) return false;
+    out.assign(std::istreambuf_iterator<char>(f), std::istreambuf_iterator<char>());
+    return !out.empty();
+}
+void write_file_atomic(const std::string &path, const std::vector<char> &data) {
+    size_t k = path.rfind('/');
+    if (k != std::string::npos) mkdir(path.substr(0, k).c_str(), 0755);
+    std::string tmp = path + ".tmp" + std::to_string((long)getpid());
+    {
+        std::ofstream f(tmp, std::ios::binary);
+        if (!f) return;
+        f.write(data.data(), (std::streamsize)data.size());
+    }
+    rename(tmp.c_str(), path.c_str());
+}
+
+up_status nvrtc_to_cubin(const std::string &src, std::vector<char> &cubin) {
     nvrtcProgram prog;
     const char *hdrs[2] = {k_up_dev_src, k_up_kparams_src};
     const char *names[2] = {"up_dev.cuh", "up_kparams.h"};
@@ -193,9 +236,26 @@ up_status compile(up_ctx *c, const std::string &src, JitKernel **out) {
     }
     size_t cs = 0;
     nvrtcGetCUBINSize(prog, &cs);
-    std::vector<char> cubin(cs);
+    cubin.resize(cs);
     nvrtcGetCUBIN(prog, cubin.data());
     nvrtcDestroyProgram(&prog);
+    return UP_OK;
+}
+
+up_status compile(up_ctx *c, const std::string &src, JitKernel **out) {
+    auto it = c->by_src.find(src);
+    if (it != c->by_src.end()) { *out = it->second.get(); return UP_OK; }
+    auto t0 = std::chrono::steady_clock::now();
+    if (const char *dump = getenv("UP_DUMP_DIR")) {
+        std::string path = std::string(dump) + "/upk_" + std::to_string(c->by_src.size()) + ".cu";
+        std::ofstream(path) << src;
+    }
+    std::vector<char> cubin;
+    const std::string cpath = cache_path(src);
+    if (cpath.empty() || !read_file(cpath, cubin)) {
+        if (up_status st = nvrtc_to_cubin(src, cubin)) return st;
+        if (!cpath.empty()) write_file_atomic(cpath, cubin);
+    }
     auto k = std::make_unique<JitKernel>();
     CU_TRY(drv.ModuleLoadData(&k->mod, cubin.data()));
     CU_TRY(drv.ModuleGetFunction(&k->fn, k->mod, "upk"));
@@ -572,6 +632,18 @@ up_status up_nvrtc_compile(const char *src, const char *cubin_path, char *log, s
         std::ofstream(cubin_path, std::ios::binary).write(cubin.data(), (std::streamsize)cs);
     }
     nvrtcDestroyProgram(&prog);
+    return UP_OK;
+}
+
+// Fill the on-disk cubin cache for a source (no GPU needed).
+up_status up_jit_prewarm(const char *src) {
+    if (!src) return fail(UP_E_INVAL, "null source");
+    const std::string cpath = cache_path(src);
+    std::vector<char> cubin;
+    if (cpath.empty()) return fail(UP_E_INVAL, "no cache directory");
+    if (read_file(cpath, cubin)) return UP_OK;
+    if (up_status st = nvrtc_to_cubin(src, cubin)) return st;
+    write_file_atomic(cpath, cubin);
     return UP_OK;
 }
 

@@ -37,7 +37,7 @@ EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_l
            "up_column_to_host_bin", "up_expr_type", "up_eval_expr", "up_sum_type", "up_sum_expr",
            "up_sum", "up_sum_combine", "up_modexp", "up_modexp_sum_type", "up_modexp_sum",
            "up_sin_taylor", "up_sin_taylor_sum", "up_check", "up_format_decimal", "up_launch_count",
-           "up_jit_ms", "up_gen_source", "up_nvrtc_compile"]
+           "up_jit_ms", "up_gen_source", "up_nvrtc_compile", "up_gen_modexp_source", "up_jit_prewarm", "up_gen_sin_source"]
 
 
 def lib():
@@ -79,6 +79,9 @@ def lib():
     L.up_jit_ms.argtypes = [P]; L.up_jit_ms.restype = c.c_double
     L.up_gen_source.argtypes = [c.c_char_p, c.c_char_p, PC, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
     L.up_nvrtc_compile.argtypes = [c.c_char_p, c.c_char_p, c.c_char_p, c.c_size_t]
+    L.up_jit_prewarm.argtypes = [c.c_char_p]
+    L.up_gen_sin_source.argtypes = [c.c_int32, c.c_int32, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
+    L.up_gen_modexp_source.argtypes = [c.c_char_p, c.c_char_p, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
     _lib = L
     return L
 
@@ -347,6 +350,23 @@ def gen_source(variant: str, expr: str, types: Sequence[tuple], n_global: int = 
     buf = ctypes.create_string_buffer(1 << 24)
     _chk(lib().up_gen_source(variant.encode(), expr.encode(), arr, len(types), n_global, buf, len(buf)))
     return buf.value.decode()
+
+
+def gen_modexp_source(exponent: int, modulus: int, base_p: int, sum: bool = False, n_global: int = 1) -> str:
+    buf = ctypes.create_string_buffer(1 << 24)
+    _chk(lib().up_gen_modexp_source(str(exponent).encode(), str(modulus).encode(), base_p, int(sum), n_global,
+                                    buf, len(buf)))
+    return buf.value.decode()
+
+
+def gen_sin_source(P: int, p: int = 9, s: int = 8, sum: bool = False, n_global: int = 1) -> str:
+    buf = ctypes.create_string_buffer(1 << 24)
+    _chk(lib().up_gen_sin_source(P, p, s, int(sum), n_global, buf, len(buf)))
+    return buf.value.decode()
+
+
+def jit_prewarm(src: str):
+    _chk(lib().up_jit_prewarm(src.encode()))
 
 
 def nvrtc_compile(src: str, cubin_path: Optional[str] = None) -> str:

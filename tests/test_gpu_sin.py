@@ -1,0 +1,73 @@
+"""GPU parity for the fixed-point Taylor sine sin_P(x) (row a9, reading Q13;
+Query 5 inputs P:L2229-2239): bit-exact vs the oracle at every P regime
+(one lane per row, and 4/8/32-lane groups = warp-cooperative, row a10)."""
+import numpy as np
+import pytest
+
+import oracle
+from gen import synth
+from tests import gpu_util as G
+
+pytestmark = pytest.mark.gpu
+
+
+def _x(n, mu, col=1):
+    return synth.normal_decimal(n, mu, 0.01, 8, config=5, column=col)
+
+
+@pytest.mark.parametrize("P,n", [(8, 300), (20, 300), (60, 300), (100, 200), (500, 40), (1000, 12), (5000, 3)])
+@pytest.mark.parametrize("mu", [0.01, 0.78, 1.56])
+def test_sin_rows_parity(P, n, mu):
+    mag, neg = _x(n, mu)
+    c = G.ctx()
+    x = c.column_from_host_bin(9, 8, mag, neg)
+    out = c.sin_taylor(x, P)
+    c.check()
+    got = c.column_to_strings(out)
+    want = oracle.sin_rows(oracle.Column(9, 8, mag, neg), P)
+    assert got == want
+
+
+def test_sin_20000_digits_sampled():
+    mag, neg = _x(2, 0.78)
+    c = G.ctx()
+    out = c.sin_taylor(c.column_from_host_bin(9, 8, mag, neg), 20000)
+    c.check()
+    assert c.column_to_strings(out) == oracle.sin_rows(oracle.Column(9, 8, mag, neg), 20000)
+
+
+@pytest.mark.parametrize("p,s,vals", [
+    (1, 0, ["0", "1", "3", "-2", "9"]),
+    (5, 2, ["0.00", "1.00", "-3.14", "9.99", "0.01"]),
+    (9, 9, ["0.000000001", "-0.999999999", "0.5"]),
+    (9, 8, ["0", "-0.00000001", "3.14159265", "-9.99999999"]),
+])
+def test_sin_edge_inputs(p, s, vals):
+    c = G.ctx()
+    for P in (max(s, 1), 40, 300):
+        out = c.sin_taylor(c.column_from_strings(p, s, vals), P)
+        c.check()
+        assert c.column_to_strings(out) == oracle.sin_rows(oracle.Column(p, s, strings=vals), P), (p, s, P)
+
+
+@pytest.mark.parametrize("P,n", [(30, 5000), (500, 300), (2000, 40)])
+def test_sin_sum_parity(P, n):
+    mag, neg = _x(n, 0.78, col=2)
+    c = G.ctx()
+    res = c.sin_taylor_sum(c.column_from_host_bin(9, 8, mag, neg), P)
+    c.check()
+    from paper_conf_icde_lixylz24_b200 import up
+    assert up.result_to_string(res, P) == oracle.sin_sum(oracle.Column(9, 8, mag, neg), P, threads=8)
+
+
+def test_sin_odd_symmetry_on_gpu():
+    mag, neg = _x(64, 0.01)      # ~16% negatives
+    c = G.ctx()
+    a = c.column_to_strings(c.sin_taylor(c.column_from_host_bin(9, 8, mag, neg), 200))
+    b = c.column_to_strings(c.sin_taylor(c.column_from_host_bin(9, 8, mag, 1 - neg), 200))
+    c.check()
+    for u, v, m in zip(a, b, mag[:, 0]):
+        if m == 0:
+            assert u == v
+        else:
+            assert u == ("-" + v if not v.startswith("-") else v[1:])

@@ -1,0 +1,62 @@
+#!/usr/bin/env python
+"""Pre-compile (NVRTC, sm_100a, no GPU needed) the specialised kernels the
+bench and the heavier tests use into libup's on-disk cubin cache, so GPU runs
+do not spend their time in NVRTC.  Purely a compile-time cache.
+
+    python tools/prewarm.py [--jobs 8]
+"""
+import argparse
+import os
+import sys
+from concurrent.futures import ProcessPoolExecutor
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def sources():
+    from gen import synth
+    from paper_conf_icde_lixylz24_b200 import up
+    out = []
+    for ws in (1, 2, 4, 8):
+        out.append(up.gen_source("sum", "c1+c2", [(17, 5), (14, 2)], 1_000_000 * ws))
+        out.append(up.gen_source("sum", "c1+c2", [(35, 5), (32, 2)], 10_000_000 * ws))
+        out.append(up.gen_source("sum", "c1*c2 - c3/c4", [(200, 50)] * 4, 12_500_000 * ws))
+        for bits in (1024, 2048):
+            N, _, _ = synth.rsa_modulus(bits)
+            out.append(up.gen_modexp_source(65537, N, len(str(N)), True, 10_000_000 * ws))
+        for P in (500, 1000, 5000, 20000):
+            out.append(up.gen_sin_source(P, 9, 8, True, 1_000_000 * ws))
+    for bits in (1024, 2048):
+        N, _, _ = synth.rsa_modulus(bits)
+        for e in (3, 65537):
+            out.append(up.gen_modexp_source(e, N, len(str(N)), False, 1))
+            out.append(up.gen_modexp_source(e, N, len(str(N)), True, 10_000_000))
+    N, _, _ = synth.rsa_modulus(512)
+    out.append(up.gen_modexp_source(65537, N, len(str(N)), True, 1001))
+    for P in (500, 1000, 5000, 20000):
+        out.append(up.gen_sin_source(P, 9, 8, False, 1))
+    out.append(up.gen_sin_source(2000, 9, 8, True, 40))
+    out.append(up.gen_sin_source(500, 9, 8, True, 300))
+    return list(dict.fromkeys(out))
+
+
+def _one(src):
+    from paper_conf_icde_lixylz24_b200 import up
+    up.jit_prewarm(src)
+    return len(src)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--jobs", type=int, default=os.cpu_count())
+    a = ap.parse_args()
+    srcs = sources()
+    with ProcessPoolExecutor(a.jobs) as ex:
+        for _ in ex.map(_one, srcs):
+            pass
+    print(f"prewarmed {len(srcs)} kernels")
+
+
+if __name__ == "__main__":
+    main()
