@@ -242,7 +242,23 @@ class Context:
         return out
 
     def column_to_strings(self, col: Column, stream=None) -> List[str]:
-        return [_fmt(v, col.s) for v in self.column_to_ints(col, stream)]
+        """Canonical decimal strings of every row (libup's formatter)."""
+        import numpy as np
+        mag = np.zeros((max(col.n, 1), col.limbs + 1), dtype=np.uint32)   # +1: keep magnitudes non-negative
+        neg = np.zeros(max(col.n, 1), dtype=np.uint8)
+        tmp = np.zeros((max(col.n, 1), col.limbs), dtype=np.uint32)
+        d = col.desc()
+        _chk(lib().up_column_to_host_bin(self.h, ctypes.byref(d), tmp.ctypes.data, neg.ctypes.data,
+                                         _stream_ptr(stream)))
+        mag[:, :col.limbs] = tmp
+        out = []
+        buf = ctypes.create_string_buffer((col.limbs + 1) * 10 + col.s + 8)
+        for i in range(col.n):
+            row = np.ascontiguousarray(mag[i])
+            _chk(lib().up_format_decimal(row.ctypes.data, col.limbs + 1, col.s, buf, len(buf)))
+            v = buf.value.decode()
+            out.append("-" + v if neg[i] and v.strip("0.") else v)
+        return out
 
     # ------------------------------------------------------------------ expressions
     def expr_type(self, expr: str, cols: Sequence[Column]):

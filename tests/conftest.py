@@ -25,3 +25,6 @@ def pytest_collection_modifyitems(config, items):
     for it in items:
         if "gpu" in it.keywords:
             it.add_marker(skip)
+
+# exact big-number tests format Python ints of up to ~20,000 digits
+sys.set_int_max_str_digits(0)
