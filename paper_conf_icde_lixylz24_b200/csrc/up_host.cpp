@@ -53,6 +53,7 @@ struct Drv {
                              CUstream, void **, void **) = nullptr;
     CUresult (*OccupancyMaxActiveBlocksPerMultiprocessor)(int *, CUfunction, int, size_t) = nullptr;
     CUresult (*GetErrorString)(CUresult, const char **) = nullptr;
+    CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
     bool ok = false;
 } drv;
 
@@ -71,6 +72,7 @@ cudaError_t load_drv() {
     UP_ENTRY("cuLaunchKernel", LaunchKernel);
     UP_ENTRY("cuOccupancyMaxActiveBlocksPerMultiprocessor", OccupancyMaxActiveBlocksPerMultiprocessor);
     UP_ENTRY("cuGetErrorString", GetErrorString);
+    UP_ENTRY("cuFuncSetAttribute", FuncSetAttribute);
 #undef UP_ENTRY
     drv.ok = true;
     return cudaSuccess;
@@ -111,6 +113,7 @@ struct JitKernel {
     int ws_slots = 0;
     int blocks_per_sm = 1;
     int threads = kThreads;
+    int dyn_smem = 0;      // dynamic shared memory per block (bytes)
     std::string src;
 };
 
@@ -304,7 +307,7 @@ up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream
     long long cap = (long long)k->blocks_per_sm * c->num_sms;
     int grid = (int)std::max(1ll, std::min(want, cap));
     void *args[] = {&P};
-    CU_TRY(drv.LaunchKernel(k->fn, grid, 1, 1, k->threads, 1, 1, 0, (CUstream)st, args, nullptr));
+    CU_TRY(drv.LaunchKernel(k->fn, grid, 1, 1, k->threads, 1, 1, (unsigned)k->dyn_smem, (CUstream)st, args, nullptr));
     c->launches++;
     return UP_OK;
 }
@@ -652,16 +655,19 @@ up_status up_jit_prewarm(const char *src) {
 
 // exported to special.cpp
 up_status up_internal_compile(up_ctx *c, const std::string &src, int rows_per_thread, int ws_slots, int threads,
-                              void **fn_out, int *blocks_per_sm) {
+                              void **fn_out, int *blocks_per_sm, int dyn_smem) {
     JitKernel *k = nullptr;
     up_status s = compile(c, src, &k);
     if (s) return s;
     k->rows_per_thread = rows_per_thread;
     k->ws_slots = ws_slots;
-    if (threads != k->threads) {
+    if (threads != k->threads || dyn_smem != k->dyn_smem) {
         k->threads = threads;
+        if (dyn_smem > 48 * 1024)
+            CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, dyn_smem));
+        k->dyn_smem = dyn_smem;
         int nb = 0;
-        CU_TRY(drv.OccupancyMaxActiveBlocksPerMultiprocessor(&nb, k->fn, threads, 0));
+        CU_TRY(drv.OccupancyMaxActiveBlocksPerMultiprocessor(&nb, k->fn, threads, (size_t)dyn_smem));
         k->blocks_per_sm = std::max(1, nb);
     }
     *fn_out = k;
