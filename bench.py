@@ -33,9 +33,18 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "tuples/sec for SELECT SUM(expr) by DECIMAL precision at 1/2/4/8 B200; % HBM/INT peak"
-# IMAD-pipe peak: 64 lanes/clk/SM (fma pipe, 2 cycles per warp instruction per
-# SMSP; B300_MICROARCH "Pipe rates") x 148 SMs x 1965 MHz max SM clock.
-IMAD_PEAK_TOPS = 64 * 148 * 1.965e9 / 1e12
+# Integer roofline for the compute-bound configs, in 32x32->64 LIMB PRODUCTS/s.
+# Every limb product needs one high-half multiply (IMAD.HI / the high half of
+# IMAD.WIDE); tools/intpipe.cu measured IMAD.HI on this B200 at 31.75
+# lanes/clk/SM (half the 60.85 of IMAD) = 9.23e12/s: the peak used below
+# (profiles/intpipe_b200_r01.json).  Fallback if the file is missing: 32
+# lanes/clk/SM x 148 SMs x 1.965 GHz.
+def _product_peak():
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "intpipe_b200_r01.json")))
+        return d["imad_hi"]["ops_per_s"], "measured IMAD.HI rate (tools/intpipe.cu, profiles/intpipe_b200_r01.json)"
+    except Exception:
+        return 32 * 148 * 1.965e9, "derived: 32 IMAD.HI lanes/clk/SM x 148 SMs x 1.965 GHz (fallback)"
 
 CONFIGS = {
     1: dict(kind="expr", name="cfg1 SUM(c1+c2) DECIMAL(17,5)+DECIMAL(14,2)", expr="c1+c2",
@@ -151,7 +160,7 @@ class ExprWorkload(Workload):
 
     def roofline(self, kernel_ms, peaks):
         if self.cfg["types"][0][0] >= 100:     # wide expressions: integer-pipe bound
-            return self._alu_roofline(kernel_ms, self.alg_imad_per_row())
+            return self._alu_roofline(kernel_ms, self.alg_products_per_row())
         alg = self.bytes_per_row * self.rows
         peak = peaks.get("hbm_gbs", 6650.0)
         ach = alg / (kernel_ms / 1e3) / 1e9
@@ -161,26 +170,26 @@ class ExprWorkload(Workload):
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks
                 else "fallback 6.65 TB/s"}
 
-    def alg_imad_per_row(self):
+    def alg_products_per_row(self):
         """limb products of c1*c2 - c3/c4 = x (L*L) + / prescale
         (L x limbs(10^(s+4))) + / (quotient limbs x L) + alignment of the
-        quotient (limbs(q) x limbs(10^(2s-(s+4)))); 2 IMAD per limb product."""
+        quotient (limbs(q) x limbs(10^(2s-(s+4))))."""
         from paper_conf_icde_lixylz24_b200 import up
         p, s = self.cfg["types"][0]
         mag = lambda k: max(1, (10 ** k).bit_length() // 32 + 1)   # noqa: E731
         L = up.limbs(p)
         nu = mag(p + s + 4)
-        products = L * L + L * mag(s + 4) + (nu - L + 1) * L + up.limbs(s + 5) * mag(s - 4)
-        return 2 * products
+        return L * L + L * mag(s + 4) + (nu - L + 1) * L + up.limbs(s + 5) * mag(s - 4)
 
-    def _alu_roofline(self, kernel_ms, imad_per_row):
-        ops = imad_per_row * self.rows
-        ach = ops / (kernel_ms / 1e3) / 1e12
-        return {"bound": "alu", "achieved": round(ach, 3), "peak": round(IMAD_PEAK_TOPS, 2), "unit": "T IMAD/s",
-                "frac": round(ach / IMAD_PEAK_TOPS, 4), "kernel_ms": round(kernel_ms, 4),
+    def _alu_roofline(self, kernel_ms, products_per_row, note=""):
+        peak, src = _product_peak()
+        ops = products_per_row * self.rows
+        ach = ops / (kernel_ms / 1e3)
+        return {"bound": "alu", "achieved": round(ach / 1e12, 4), "peak": round(peak / 1e12, 4),
+                "unit": "T limb-products/s", "frac": round(ach / peak, 4), "kernel_ms": round(kernel_ms, 4),
                 "alg_ops_per_launch": ops,
-                "alg_unit": f"{imad_per_row} IMAD-pipe ops/row (2 per 32x32 limb product) x {self.rows} rows",
-                "peak_source": "derived: 64 IMAD lanes/clk/SM x 148 SMs x 1965 MHz (DESIGN.md)"}
+                "alg_unit": f"{products_per_row} 32x32->64 limb products/row x {self.rows} rows" + note,
+                "peak_source": src}
 
     def host_for_oracle(self):
         import numpy as np
@@ -226,7 +235,8 @@ class ModexpWorkload(ExprWorkload):
     def roofline(self, kernel_ms, peaks):
         n = (self.N.bit_length() + 31) // 32
         montmuls = (self.e.bit_length() - 1) + bin(self.e).count("1") - 1 + 2   # squarings + multiplies + in/out
-        return self._alu_roofline(kernel_ms, 2 * montmuls * (2 * n * n + n))
+        return self._alu_roofline(kernel_ms, montmuls * (2 * n * n + n),
+                                  f"; {montmuls} Montgomery products x (2n^2+n), n = {n}")
 
     def oracle_sum(self, ocols, n, threads):
         import oracle
@@ -256,16 +266,17 @@ class SinWorkload(ExprWorkload):
         self.LA = up.limbs(self.P)
         self.e2e_cols = [up.Column(9, 8, self.rows)]
         self.cfg = dict(cfg, types=[(9, 8)])
-        # mean number of Taylor terms (for the algorithmic op count), from a sample
+        # active-limb sum per row, from a sample of rows
         import numpy as np
-        ks = []
-        for m in mag[: 256, 0].tolist():
-            t, k = m * 10 ** (self.Pd - 8), 1
+        acts = []
+        for m in mag[: 128, 0].tolist():
+            t, k, a = m * 10 ** (self.Pd - 8), 1, 0
             while t:
+                a += (t.bit_length() + 31) // 32
                 t = t * m * m // (10 ** 16 * (2 * k) * (2 * k + 1))
                 k += 1
-            ks.append(k - 1)
-        self.mean_terms = float(np.mean(ks))
+            acts.append(a)
+        self.active_limb_terms = float(np.mean(acts))
 
     def kernel(self, out):
         self.ctx.sin_taylor_sum(self.cols[0], self.Pd, self.n_global, out=out)
@@ -274,14 +285,11 @@ class SinWorkload(ExprWorkload):
         self.ctx.sin_taylor_sum(self.e2e_cols[0], self.Pd, self.n_global, out=out)
 
     def roofline(self, kernel_ms, peaks):
-        from paper_conf_icde_lixylz24_b200 import up
-        W = up.limbs(self.Pd + 23)
-        # per term and limb: x m_x^2 (2 limb products = 4 IMAD) + 3 short-division
-        # steps (64x64 high product ~4 IMAD + q*d 1 IMAD each) = 19 IMAD-pipe ops
-        per_row = int(self.mean_terms * W * 19)
-        r = self._alu_roofline(kernel_ms, per_row)
-        r["alg_unit"] += f"; mean {self.mean_terms:.1f} terms x {W} limbs x 19"
-        return r
+        # per active limb-term: t x m_x^2 (2 limb products) + 3 short-division
+        # steps (one 32x32->64 reciprocal product each) = 5 limb products
+        per_row = int(round(self.active_limb_terms * 5))
+        return self._alu_roofline(kernel_ms, per_row,
+                                  f"; mean active-limb sum {self.active_limb_terms:.0f} per row x 5")
 
     def oracle_sum(self, ocols, n, threads):
         import oracle

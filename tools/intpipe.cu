@@ -74,6 +74,24 @@ __global__ void k_rowmac(unsigned *out, unsigned m, unsigned c) {
     out[blockIdx.x * blockDim.x + threadIdx.x] = r0 ^ r1 ^ r2 ^ r3;
 }
 
+// 32x32->64 products: one mul.wide per step vs a mul.lo + mul.hi pair
+__global__ void k_mulwide(unsigned *out, unsigned m, unsigned c) {
+    unsigned a0 = threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5, a6 = a0 + 6, a7 = a0 + 7;
+#define OP(x) { unsigned long long r; asm volatile("mul.wide.u32 %0, %1, %2;" : "=l"(r) : "r"(x), "r"(m)); \
+                x = (unsigned)r ^ (unsigned)(r >> 32); }
+    for (int i = 0; i < ITERS; ++i) { CHAIN8(OP) }
+#undef OP
+    out[blockIdx.x * blockDim.x + threadIdx.x] = a0 ^ a1 ^ a2 ^ a3 ^ a4 ^ a5 ^ a6 ^ a7;
+}
+__global__ void k_mullohi(unsigned *out, unsigned m, unsigned c) {
+    unsigned a0 = threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5, a6 = a0 + 6, a7 = a0 + 7;
+#define OP(x) { unsigned lo, hi; asm volatile("mul.lo.u32 %0, %2, %3;\n\tmul.hi.u32 %1, %2, %3;" : "=r"(lo), "=r"(hi) : "r"(x), "r"(m)); \
+                x = lo ^ hi; }
+    for (int i = 0; i < ITERS; ++i) { CHAIN8(OP) }
+#undef OP
+    out[blockIdx.x * blockDim.x + threadIdx.x] = a0 ^ a1 ^ a2 ^ a3 ^ a4 ^ a5 ^ a6 ^ a7;
+}
+
 template <typename K>
 double run(K kern, const char *name, double ops_per_thread, int sms, double &lanes_per_clk_sm, double &clk_ghz) {
     unsigned *out;
@@ -120,6 +138,10 @@ int main() {
     printf(", \"iadd\": {\"ops_per_s\": %.4e, \"lanes_per_clk_sm_at_max_clock\": %.2f}", v, l);
     v = run(k_rowmac, "row_mac", 8.0 * (ITERS / 2), sms, l, g);
     printf(", \"mad_cc_chain\": {\"ops_per_s\": %.4e, \"lanes_per_clk_sm_at_max_clock\": %.2f, \"note\": \"PTX mad.lo/hi.cc ops (2 per limb product)\"}", v, l);
+    v = run(k_mulwide, "mul_wide", 8.0 * ITERS, sms, l, g);
+    printf(", \"mul_wide_products\": {\"ops_per_s\": %.4e, \"lanes_per_clk_sm_at_max_clock\": %.2f}", v, l);
+    v = run(k_mullohi, "mul_lohi", 8.0 * ITERS, sms, l, g);
+    printf(", \"mul_lo_hi_products\": {\"ops_per_s\": %.4e, \"lanes_per_clk_sm_at_max_clock\": %.2f}", v, l);
     printf(", \"clock_ghz_attr\": %.3f}\n", g);
     return 0;
 }
