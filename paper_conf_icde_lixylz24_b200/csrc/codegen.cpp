@@ -237,4 +237,194 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     return k.str();
 }
 
+
+// ---------------------------------------------------------------------------
+// Wide SUM regime (rows a10/a11 at ~40+ limbs, cfg3 DECIMAL(500..1000,...)):
+// SELECT SUM(sum_t +-term_t) = sum_t +-10^(s_out - s_t) SUM(term_t) exactly
+// (alignment is an exact x10^k and SUM is linear), so each term is summed on
+// its own and the constant alignment is applied once at the end.  Terms:
+// c_i, c_i*c_j, c_i/c_j.  One warp per row; a product is summed as exact
+// column sums (no per-row carry normalisation); a quotient runs a
+// warp-cooperative Knuth D on shared-memory operands.
+namespace {
+
+struct WTerm {
+    int kind;   // 0 col, 1 mul, 2 div
+    int sign;   // +1 / -1
+    const Node *n;
+    int ca = -1, cb = -1;
+};
+
+bool flatten(const Node *n, int sign, std::vector<WTerm> &out) {
+    switch (n->op) {
+    case Op::Add: return flatten(n->l.get(), sign, out) && flatten(n->r.get(), sign, out);
+    case Op::Sub: return flatten(n->l.get(), sign, out) && flatten(n->r.get(), -sign, out);
+    case Op::Neg: return flatten(n->l.get(), -sign, out);
+    case Op::Col: out.push_back({0, sign, n, n->col, -1}); return true;
+    case Op::Mul:
+        if (n->l->op == Op::Col && n->r->op == Op::Col) { out.push_back({1, sign, n, n->l->col, n->r->col}); return true; }
+        return false;
+    case Op::Div:
+        if (n->l->op == Op::Col && n->r->op == Op::Col) { out.push_back({2, sign, n, n->l->col, n->r->col}); return true; }
+        return false;
+    default: return false;
+    }
+}
+
+}  // namespace
+
+std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &cols, int LA, GenInfo &info) {
+    std::vector<WTerm> terms;
+    if (!flatten(root, 1, terms) || terms.empty() || terms.size() > 8) return "";
+    std::vector<bool> used(cols.size(), false);
+    used_columns(root, used);
+    constexpr int NW = 8;
+    std::ostringstream k;
+    k << "// generated by libup codegen (wide SUM regime): " << canonical(root) << "  type (" << root->p << "," << root->s
+      << ") LA=" << LA << "\n";
+    k << "#include \"up_dev.cuh\"\n#include \"up_wide.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
+    // smem plan (in u32 words; u64 slot arrays first for alignment)
+    int slot_words = 0;
+    std::vector<int> slot_off(terms.size()), slot_n(terms.size());
+    for (size_t t = 0; t < terms.size(); ++t) {
+        const WTerm &w = terms[t];
+        int ns = 0;
+        if (w.kind == 0) ns = cols[(size_t)w.ca].limbs + 1;
+        if (w.kind == 1) ns = cols[(size_t)w.ca].limbs + cols[(size_t)w.cb].limbs + 2;
+        if (w.kind == 2) ns = w.n->L + 1;
+        slot_off[t] = slot_words;
+        slot_n[t] = ns;
+        slot_words += 2 * ns;   // pos and neg u64 arrays (counted in u64 units here)
+    }
+    if (slot_words * 2 > 16000) return "";
+    // per-warp scratch: staged columns + magnitude copies + division scratch
+    int stage = 0;
+    std::vector<int> stage_off(cols.size(), -1);
+    for (size_t c = 0; c < cols.size(); ++c)
+        if (used[c]) { stage_off[c] = stage; stage += cols[c].limbs; }
+    int scratch = 0;
+    int magA = 0, magB = 0, divU = 0, divS = 0, divQ = 0, maxA = 0, maxB = 0;
+    for (auto &w : terms) {
+        if (w.kind == 0) continue;
+        maxA = std::max(maxA, cols[(size_t)w.ca].limbs);
+        maxB = std::max(maxB, cols[(size_t)w.cb].limbs);
+    }
+    magA = scratch; scratch += maxA;
+    magB = scratch; scratch += maxB;
+    int maxNU = 0, maxNS = 0, maxNQ = 0;
+    for (auto &w : terms) {
+        if (w.kind != 2) continue;
+        const Node *A = w.n->l.get(), *B = w.n->r.get();
+        const int NU = mag_limbs_of_pow10(A->p + B->s + 4);
+        const int NV = B->L;
+        maxNU = std::max(maxNU, NU);
+        maxNS = std::max(maxNS, NU + NV + 1 + NV);
+        maxNQ = std::max(maxNQ, w.n->L);
+    }
+    divU = scratch; scratch += maxNU;
+    divS = scratch; scratch += maxNS;
+    divQ = scratch; scratch += maxNQ;
+    const int per_warp = stage + scratch;
+    const int smem_bytes = slot_words * 8 + NW * per_warp * 4;
+    if (smem_bytes > 200 * 1024) return "";
+    info.rows_per_thread = 1;
+    info.ws_slots = slot_words;
+    info.dyn_smem = smem_bytes;
+    info.threads = NW * 32;
+    info.rows_per_block = NW;
+
+    k << "extern \"C\" __global__ void __launch_bounds__(" << NW * 32 << ") upk(const up_kparams P) {\n";
+    k << "    constexpr int NW = " << NW << ", PER_WARP = " << per_warp << ", SLOTS = " << slot_words << ";\n";
+    k << "    extern __shared__ u64 smem64[];\n";
+    k << "    u64 *slots = smem64;\n";
+    k << "    u32 *wbase = reinterpret_cast<u32 *>(smem64 + SLOTS);\n";
+    k << "    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;\n";
+    k << "    u32 *my = wbase + warp * PER_WARP;\n";
+    k << "    for (int i = tid; i < SLOTS; i += blockDim.x) slots[i] = 0ull;\n";
+    k << "    u32 fl = 0;\n";
+    k << "    const long long n = P.n;\n";
+    k << "    for (long long r0 = (long long)blockIdx.x * NW; r0 < n; r0 += (long long)gridDim.x * NW) {\n";
+    k << "        __syncthreads();\n";
+    // cooperative, sector-coalesced staging: 8 consecutive threads read 8 rows of one plane
+    for (size_t c = 0; c < cols.size(); ++c) {
+        if (!used[c]) continue;
+        const int Lc = cols[c].limbs;
+        k << "        for (int idx = tid; idx < " << Lc << " * NW; idx += blockDim.x) { const int j = idx / NW, w = idx % NW;\n"
+             "            const long long row = r0 + w;\n"
+             "            wbase[w * PER_WARP + " << stage_off[c] << " + j] = row < n ? __ldcs(P.col[" << c << "] + (long long)j * P.ld[" << c << "] + row) : 0u; }\n";
+    }
+    k << "        __syncthreads();\n";
+    k << "        if (r0 + warp < n) {\n";
+    for (size_t t = 0; t < terms.size(); ++t) {
+        const WTerm &w = terms[t];
+        const std::string pos = "(slots + " + std::to_string(slot_off[t]) + ")";
+        const std::string neg = "(slots + " + std::to_string(slot_off[t] + slot_n[t]) + ")";
+        k << "            { // term " << t << ": " << (w.sign > 0 ? "+" : "-") << canonical(w.n) << "\n";
+        if (w.kind == 0) {
+            const int Lc = cols[(size_t)w.ca].limbs;
+            k << "              const u32 *x = my + " << stage_off[(size_t)w.ca] << ";\n";
+            k << "              for (int j = lane; j < " << Lc << "; j += 32) if (x[j]) atomicAdd(&" << pos << "[j], (u64)x[j]);\n";
+            k << "              if (lane == 0 && (x[" << Lc - 1 << "] >> 31)) atomicAdd(&" << neg << "[" << Lc << "], 1ull);\n";
+        } else {
+            const int La = cols[(size_t)w.ca].limbs, Lb = cols[(size_t)w.cb].limbs;
+            k << "              u32 *A = my + " << magA << ", *B = my + " << magB << ";\n";
+            k << "              for (int j = lane; j < " << La << "; j += 32) A[j] = my[" << stage_off[(size_t)w.ca] << " + j];\n";
+            k << "              for (int j = lane; j < " << Lb << "; j += 32) B[j] = my[" << stage_off[(size_t)w.cb] << " + j];\n";
+            k << "              __syncwarp();\n";
+            k << "              const u32 sa = wide::to_mag<" << La << ">(A), sb = wide::to_mag<" << Lb << ">(B);\n";
+            if (w.kind == 1) {
+                k << "              u64 *acc = (sa ^ sb) ? " << neg << " : " << pos << ";\n";
+                if (La == Lb) k << "              wide::colsum_product_sq<" << La << ">(A, B, acc);\n";
+                else k << "              wide::colsum_product<" << La << "," << Lb << ">(A, B, acc);\n";
+            } else {
+                const Node *An = w.n->l.get(), *Bn = w.n->r.get();
+                const int kk = Bn->s + 4;
+                const int NU = mag_limbs_of_pow10(An->p + kk);
+                HBig c = HBig::pow10(kk);
+                const int LC = (int)c.w.size();
+                const int NQ = w.n->L;
+                std::vector<uint32_t> cw(c.w.begin(), c.w.end());
+                k << "              const u32 KC[" << LC << "] = " << limbs_init(cw) << ";\n";
+                k << "              u32 *U = my + " << divU << ", *Q = my + " << divQ << ";\n";
+                k << "              wide::mul_const<" << La << "," << LC << "," << NU << ">(A, KC, U);\n";
+                k << "              u32 f = wide::divq<" << NU << "," << Lb << "," << NQ << ">(U, B, Q, my + " << divS << ");\n";
+                std::vector<uint32_t> bw = HBig::pow10(w.n->p).twos(NQ, false);
+                k << "              const u32 BOUND[" << NQ << "] = " << limbs_init(bw) << ";\n";
+                k << "              if (!f && !wide::lt_bound<" << NQ << ">(Q, BOUND)) f = F_OVERFLOW;\n";
+                k << "              fl |= f;\n";
+                k << "              if (!f) { u64 *acc = (sa ^ sb) ? " << neg << " : " << pos << ";\n"
+                     "                for (int j = lane; j < " << NQ << "; j += 32) if (Q[j]) atomicAdd(&acc[j], (u64)Q[j]); }\n";
+            }
+        }
+        k << "              __syncwarp();\n            }\n";
+    }
+    k << "        }\n";
+    k << "    }\n";
+    k << "    if (fl) atomicOr(P.flags, fl);\n";
+    // commit all slots; last block combines
+    k << "    __syncthreads();\n";
+    k << "    for (int i = tid; i < SLOTS; i += blockDim.x) if (slots[i]) atomicAdd(&P.ws[i], slots[i]);\n";
+    k << "    __threadfence();\n    __syncthreads();\n";
+    k << "    __shared__ u32 s_last;\n";
+    k << "    if (tid == 0) s_last = (atomicAdd(P.ticket, 1u) == gridDim.x - 1) ? 1u : 0u;\n";
+    k << "    __syncthreads();\n    if (!s_last) return;\n    __threadfence();\n";
+    k << "    for (int i = tid; i < SLOTS; i += blockDim.x) slots[i] = atomicExch(&P.ws[i], 0ull);\n";
+    k << "    __syncthreads();\n";
+    k << "    if (tid == 0) {\n";
+    k << "        *P.ticket = 0u;\n";
+    k << "        u32 acc[" << LA << "];\n        for (int j = 0; j < " << LA << "; ++j) acc[j] = 0u;\n";
+    for (size_t t = 0; t < terms.size(); ++t) {
+        const WTerm &w = terms[t];
+        const int kt = root->s - w.n->s;
+        HBig c = HBig::pow10(kt);
+        std::vector<uint32_t> cw(c.w.begin(), c.w.end());
+        k << "        { const u32 KT[" << cw.size() << "] = " << limbs_init(cw) << ";\n";
+        k << "          wide::wide_final(slots + " << slot_off[t] << ", slots + " << slot_off[t] + slot_n[t] << ", "
+          << slot_n[t] << ", KT, " << cw.size() << ", " << w.sign << ", " << LA << ", acc); }\n";
+    }
+    k << "        for (int j = 0; j < " << LA << "; ++j) P.result[j] = acc[j];\n";
+    k << "    }\n";
+    k << "}\n";
+    return k.str();
+}
 }  // namespace uph

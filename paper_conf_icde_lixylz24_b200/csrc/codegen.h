@@ -15,9 +15,14 @@ struct GenOpts {
 struct GenInfo {
     int rows_per_thread = 1;
     int ws_slots = 0;
+    int dyn_smem = 0;        // dynamic shared memory per block (bytes)
+    int threads = 256;
+    int rows_per_block = 0;  // > 0: rows handled per block-iteration (warp-per-row kernels)
 };
 
 std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, const GenOpts &opt, GenInfo &info);
+// wide SUM regime (warp per row); "" if the expression does not fit it
+std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &cols, int LA, GenInfo &info);
 
 // modexp / sin_taylor specialisations (special.cpp)
 struct ModexpPlan {

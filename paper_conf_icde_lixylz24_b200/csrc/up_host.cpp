@@ -105,6 +105,7 @@ up_status fail(up_status st, const char *fmt, ...) {
 
 constexpr int kThreads = 256;
 constexpr int kWsSlots = 1 << 16;
+constexpr int kWideMinLimbs = 40;   // per-thread registers stop scaling beyond this
 
 struct JitKernel {
     CUmodule mod = nullptr;
@@ -114,6 +115,7 @@ struct JitKernel {
     int blocks_per_sm = 1;
     int threads = kThreads;
     int dyn_smem = 0;      // dynamic shared memory per block (bytes)
+    int rows_per_block = 0;  // > 0: warp-per-row kernels (rows per block-iteration)
     std::string src;
 };
 
@@ -200,6 +202,7 @@ std::string cache_path(const std::string &src) {
     for (const char *o : kNvrtcOpts) h = fnv1a(o, h);
     h = fnv1a(k_up_dev_src, h);
     h = fnv1a(k_up_kparams_src, h);
+    h = fnv1a(k_up_wide_src, h);
     char name[64];
     snprintf(name, sizeof name, "/%016llx.cubin", (unsigned long long)h);
     return d + name;
@@ -224,9 +227,9 @@ void write_file_atomic(const std::string &path, const std::vector<char> &data) {
 
 up_status nvrtc_to_cubin(const std::string &src, std::vector<char> &cubin) {
     nvrtcProgram prog;
-    const char *hdrs[2] = {k_up_dev_src, k_up_kparams_src};
-    const char *names[2] = {"up_dev.cuh", "up_kparams.h"};
-    if (nvrtcCreateProgram(&prog, src.c_str(), "upk.cu", 2, hdrs, names) != NVRTC_SUCCESS)
+    const char *hdrs[3] = {k_up_dev_src, k_up_kparams_src, k_up_wide_src};
+    const char *names[3] = {"up_dev.cuh", "up_kparams.h", "up_wide.cuh"};
+    if (nvrtcCreateProgram(&prog, src.c_str(), "upk.cu", 3, hdrs, names) != NVRTC_SUCCESS)
         return fail(UP_E_NVRTC, "nvrtcCreateProgram failed");
     nvrtcResult r = nvrtcCompileProgram(prog, (int)(sizeof kNvrtcOpts / sizeof kNvrtcOpts[0]), kNvrtcOpts);
     if (r != NVRTC_SUCCESS) {
@@ -302,7 +305,7 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
 }
 
 up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream_t st) {
-    long long per_block = (long long)k->threads * k->rows_per_thread;
+    long long per_block = k->rows_per_block > 0 ? k->rows_per_block : (long long)k->threads * k->rows_per_thread;
     long long want = (n + per_block - 1) / per_block;
     long long cap = (long long)k->blocks_per_sm * c->num_sms;
     int grid = (int)std::max(1ll, std::min(want, cap));
@@ -327,13 +330,30 @@ up_status expr_kernel(up_ctx *c, const char *expr, const up_column *cols, int nc
     o.sum = sum;
     o.LA = LA;
     GenInfo info;
-    std::string src = gen_expr_kernel(t.root.get(), t.types, o, info);
+    std::string src;
+    // wide SUM regime: warp per row, linear decomposition into summed terms
+    if (sum && max_limbs(t.root.get()) >= kWideMinLimbs && LA <= 512 && !getenv("UP_NO_WIDE"))
+        src = gen_wide_sum_kernel(t.root.get(), t.types, LA, info);
+    if (src.empty()) {
+        info = GenInfo();
+        src = gen_expr_kernel(t.root.get(), t.types, o, info);
+    }
     if (sum && info.ws_slots > kWsSlots) return fail(UP_E_UNSUPPORTED, "SUM too wide (%d slots)", info.ws_slots);
     JitKernel *k = nullptr;
     s = compile(c, src, &k);
     if (s) return s;
     k->rows_per_thread = info.rows_per_thread;
     k->ws_slots = info.ws_slots;
+    k->rows_per_block = info.rows_per_block;
+    if (info.threads != k->threads || info.dyn_smem != k->dyn_smem) {
+        k->threads = info.threads;
+        if (info.dyn_smem > 48 * 1024)
+            CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, info.dyn_smem));
+        k->dyn_smem = info.dyn_smem;
+        int nb = 0;
+        CU_TRY(drv.OccupancyMaxActiveBlocksPerMultiprocessor(&nb, k->fn, k->threads, (size_t)k->dyn_smem));
+        k->blocks_per_sm = std::max(1, nb);
+    }
     c->by_key[key] = k;
     *out = k;
     return UP_OK;
@@ -606,7 +626,10 @@ up_status up_gen_source(const char *variant, const char *expr, const up_column *
     const long long N = n_global > 0 ? n_global : (ncols ? cols[0].n : 0);
     o.LA = o.sum ? limbs_for_precision(sum_precision(t.root->p, N)) : 0;
     GenInfo info;
-    std::string src = gen_expr_kernel(t.root.get(), t.types, o, info);
+    std::string src;
+    if (o.sum && max_limbs(t.root.get()) >= kWideMinLimbs && o.LA <= 512 && !getenv("UP_NO_WIDE"))
+        src = gen_wide_sum_kernel(t.root.get(), t.types, o.LA, info);
+    if (src.empty()) src = gen_expr_kernel(t.root.get(), t.types, o, info);
     if (src.size() + 1 > len) return fail(UP_E_NOMEM, "need %zu bytes", src.size() + 1);
     memcpy(buf, src.c_str(), src.size() + 1);
     return UP_OK;
@@ -614,9 +637,9 @@ up_status up_gen_source(const char *variant, const char *expr, const up_column *
 
 up_status up_nvrtc_compile(const char *src, const char *cubin_path, char *log, size_t len) {
     nvrtcProgram prog;
-    const char *hdrs[2] = {k_up_dev_src, k_up_kparams_src};
-    const char *names[2] = {"up_dev.cuh", "up_kparams.h"};
-    if (nvrtcCreateProgram(&prog, src, "upk.cu", 2, hdrs, names) != NVRTC_SUCCESS)
+    const char *hdrs[3] = {k_up_dev_src, k_up_kparams_src, k_up_wide_src};
+    const char *names[3] = {"up_dev.cuh", "up_kparams.h", "up_wide.cuh"};
+    if (nvrtcCreateProgram(&prog, src, "upk.cu", 3, hdrs, names) != NVRTC_SUCCESS)
         return fail(UP_E_NVRTC, "nvrtcCreateProgram failed");
     std::vector<const char *> opts(kNvrtcOpts, kNvrtcOpts + sizeof kNvrtcOpts / sizeof kNvrtcOpts[0]);
     opts.push_back("-Xptxas=-v");

@@ -1,0 +1,79 @@
+"""GPU parity of the wide SUM regime (warp per row, rows a10/a11): cfg3's
+SUM(c1*c2 - c3/c4) at DECIMAL(200,50) / (500,75) / (1000,100) and other
+linear combinations of column, product and quotient terms, vs the oracle."""
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from gen import synth
+from tests import gpu_util as G
+
+pytestmark = pytest.mark.gpu
+
+
+def _sum(expr, types, n, lead=(), seed=synth.SEED):
+    host = G.gen_cols(n, types, config=3, nonzero_lead_cols=lead, seed=seed)
+    want, P, S = oracle.eval_sum(expr, G.to_oracle(host, types), threads=8)
+    got, gP, gS = G.gpu_sum_string(expr, G.to_gpu(host, types))
+    assert (gP, gS) == (P, S)
+    return got, want
+
+
+@pytest.mark.parametrize("p,s", [(200, 50), (500, 75), (1000, 100)])
+@pytest.mark.parametrize("n", [1, 9, 1000])
+def test_cfg3_wide_sum_parity(p, s, n):
+    got, want = _sum("c1*c2 - c3/c4", [(p, s)] * 4, n, lead=(3,))
+    assert got == want
+
+
+@pytest.mark.parametrize("expr,types,lead", [
+    ("c1*c2 + c3", [(300, 20), (300, 40), (330, 60)], ()),
+    ("-c1*c1 - c2/c3 + c1", [(400, 10), (380, 5), (350, 100)], (2,)),
+    ("c1/c2 - c3*c4", [(450, 0), (300, 0), (420, 30), (400, 30)], (1,)),
+    ("c1*c2", [(600, 200), (300, 100)], ()),
+])
+def test_wide_linear_combinations(expr, types, lead):
+    got, want = _sum(expr, types, 777, lead=lead)
+    assert got == want
+
+
+def test_wide_edge_values_and_flags():
+    c = G.ctx()
+    p = 400
+    big = str(10 ** p - 1)
+    vals1 = [big, "-" + big, "0", "1", "-1", big]
+    vals2 = ["-" + big, big, big, "7", "-" + big, "0"]
+    ga = c.column_from_strings(p, 0, vals1)
+    gb = c.column_from_strings(p, 0, vals2)
+    oa, ob = oracle.Column(p, 0, strings=vals1), oracle.Column(p, 0, strings=vals2)
+    from paper_conf_icde_lixylz24_b200 import up
+    res = c.sum_expr("c1*c2 - c2", [ga, gb])
+    c.check()
+    assert up.result_to_string(res, 0) == oracle.eval_sum("c1*c2 - c2", [oa, ob])[0]
+    # division by zero in one row sets the flag
+    c.sum_expr("c1/c2", [ga, gb])
+    with pytest.raises(up.UpError) as ei:
+        c.check()
+    assert ei.value.name in ("DIVZERO", "OVERFLOW")
+
+
+def test_wide_and_per_thread_paths_agree(monkeypatch):
+    """p=200 sits on the regime boundary: the per-thread fused kernel
+    (UP_NO_WIDE) and the wide kernel must give the same bits."""
+    types = [(200, 50)] * 4
+    host = G.gen_cols(500, types, config=3, nonzero_lead_cols=(3,), seed=7)
+    from paper_conf_icde_lixylz24_b200 import up
+    c1 = up.Context(0)
+    a, _, _ = (None, None, None)
+    cols = [c1.column_from_host_bin(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
+    P, S, LA = c1.sum_type("c1*c2 - c3/c4", cols)
+    wide = up.result_to_string(c1.sum_expr("c1*c2 - c3/c4", cols), S)
+    c1.check()
+    monkeypatch.setenv("UP_NO_WIDE", "1")
+    c2 = up.Context(0)
+    cols2 = [c2.column_from_host_bin(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
+    narrow = up.result_to_string(c2.sum_expr("c1*c2 - c3/c4", cols2), S)
+    c2.check()
+    assert wide == narrow
