@@ -87,7 +87,7 @@ __device__ __forceinline__ void colsum_product(const u32 *a, const u32 *b, u64 *
 // a shuffled 64-bit carry and a ballot-resolved 1-bit carry between lanes.
 template <int LA, int LC, int NU>
 __device__ __forceinline__ void mul_const(const u32 *a, const u32 (&c)[LC], u32 *u) {
-    constexpr int CH = (NU + 31) / 32;
+    constexpr int CH = (NU + 31) / 32 < 2 ? 2 : (NU + 31) / 32;   // >= 2: the 64-bit carry spans two limbs
     const Grp<32> g;
     u32 limb[CH];
     u64 carry = 0;   // local running carry (< 2^40)
@@ -112,16 +112,11 @@ __device__ __forceinline__ void mul_const(const u32 *a, const u32 (&c)[LC], u32 
     }
     // carry out of this chunk goes to the next lane's lowest limbs
     const u32 c0 = g.up1((u32)carry), c1 = g.up1((u32)(carry >> 32));
-    u32 cy;
     limb[0] = add_cc(limb[0], c0);
-    if (CH > 1) {
-        limb[CH > 1 ? 1 : 0] = addc_cc(limb[CH > 1 ? 1 : 0], c1);
+    limb[1] = addc_cc(limb[1], c1);
 #pragma unroll
-        for (int t = 2; t < CH; ++t) limb[t] = addc_cc(limb[t], 0u);
-        cy = addc(0u, 0u);
-    } else {
-        cy = addc(0u, 0u) + c1;   // CH == 1: c1 lands one limb up (next lane); sizing keeps it 0 here
-    }
+    for (int t = 2; t < CH; ++t) limb[t] = addc_cc(limb[t], 0u);
+    const u32 cy = addc(0u, 0u);
     chunk_inc(limb, g.carry_in(cy != 0u, chunk_all_ones(limb), 0u));
 #pragma unroll
     for (int t = 0; t < CH; ++t) {
