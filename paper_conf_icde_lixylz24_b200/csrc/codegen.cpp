@@ -302,7 +302,7 @@ std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &co
     std::vector<int> stage_off(cols.size(), -1);
     for (size_t c = 0; c < cols.size(); ++c)
         if (used[c]) { stage_off[c] = stage; stage += cols[c].limbs; }
-    int scratch = 0;
+    int scratch = stage;   // scratch follows the staged columns in the warp's slice
     int magA = 0, magB = 0, divU = 0, divS = 0, divQ = 0, maxA = 0, maxB = 0;
     for (auto &w : terms) {
         if (w.kind == 0) continue;
@@ -324,7 +324,7 @@ std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &co
     divU = scratch; scratch += maxNU;
     divS = scratch; scratch += maxNS;
     divQ = scratch; scratch += maxNQ;
-    const int per_warp = stage + scratch;
+    const int per_warp = scratch;
     const int smem_bytes = slot_words * 8 + NW * per_warp * 4;
     if (smem_bytes > 200 * 1024) return "";
     info.rows_per_thread = 1;
