@@ -105,7 +105,7 @@ up_status fail(up_status st, const char *fmt, ...) {
 
 constexpr int kThreads = 256;
 constexpr int kWsSlots = 1 << 16;
-constexpr int kWideMinLimbs = 40;   // per-thread registers stop scaling beyond this
+constexpr int kWideMinLimbs = 257;  // warp-per-row only beyond this (per-thread measured faster at p <= 1000)
 
 struct JitKernel {
     CUmodule mod = nullptr;
