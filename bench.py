@@ -15,8 +15,8 @@ kernel (+ NCCL all-gather of the partials and the exact combine kernel when
 N > 1).  Inputs are seeded synthetic columns (gen/).  For N > 1 rows are
 sharded (weak scaling: every rank owns `rows` rows; typing uses the global
 row count).  Reported with it: `e2e` (same metric through the C ABI from
-pinned HOST buffers: H2D + ingestion + SUM + D2H of the result in the timed
-region), `roofline` of the fused kernel, `cpu_baseline` (the CPU oracle as it
+pinned HOST buffers in the paper's compact row format: H2D + ingestion + SUM
++ D2H of the result in the timed region), `roofline` of the fused kernel, `cpu_baseline` (the CPU oracle as it
 stands on a bounded sample), NVML clocks during the timed region, and
 `gpu_launches`.  `--impl reference` times the CPU oracle (the reference arm).
 """
@@ -151,9 +151,23 @@ class ExprWorkload(Workload):
     def kernel(self, out):
         self.ctx.sum_expr(self.cfg["expr"], self.cols, self.n_global, out=out)
 
+    def e2e_host_buffers(self):
+        """Pinned host copies of the inputs in the paper's compact row format
+        (P:L843-873): Lb bytes per row, what a scan would hand to the GPU."""
+        import numpy as np
+        import torch
+        from gen import synth
+        bufs = []
+        for (mag, neg), (p, s) in zip(self.raw, self.cfg["types"]):
+            cb = synth.to_compact(mag.cpu().numpy().view(np.uint32), neg.cpu().numpy(), p)
+            t = torch.empty(cb.shape, dtype=torch.uint8, pin_memory=True)
+            t.copy_(torch.from_numpy(cb))
+            bufs.append(t)
+        return bufs
+
     def e2e_ingest(self, host):
-        for (hm, hn), (p, s), col in zip(host, self.cfg["types"], self.e2e_cols):
-            self.ctx.column_from_host_bin(p, s, hm, hn, out=col)
+        for hb, (p, s), col in zip(host, self.cfg["types"], self.e2e_cols):
+            self.ctx.column_from_compact(p, s, hb, n=self.rows, out=col)
 
     def e2e_kernel(self, out):
         self.ctx.sum_expr(self.cfg["expr"], self.e2e_cols, self.n_global, out=out)
@@ -488,13 +502,7 @@ def main():
             pass
 
     # ---- e2e through the C ABI from pinned host buffers
-    host = []
-    for mag, neg in wl.raw:
-        hm = torch.empty(mag.shape, dtype=torch.int32, pin_memory=True)
-        hn = torch.empty(neg.shape, dtype=torch.uint8, pin_memory=True)
-        hm.copy_(mag)
-        hn.copy_(neg)
-        host.append((hm, hn))
+    host = wl.e2e_host_buffers()
     torch.cuda.synchronize()
     res_host = torch.empty(LA, dtype=torch.int32, pin_memory=True)
 
@@ -528,7 +536,7 @@ def main():
         ems = float(t.item())
     ctx.check()
     assert up.format_decimal(res_host.tolist(), wl.S) == result, "e2e result differs from the resident run"
-    h2d = sum(hm.numel() * 4 + hn.numel() for hm, hn in host)
+    h2d = sum(hb.numel() for hb in host)
     e2e = {"value": n_global / (ems / K2 / 1e3), "unit": "tuples/s", "h2d_bytes_per_step": h2d,
            "d2h_bytes_per_step": LA * 4, "ms_per_step": ems / K2}
 

@@ -200,3 +200,22 @@ def to_ints(mag: np.ndarray, neg: np.ndarray):
         v = words_to_int(mag[i])
         out.append(-v if neg[i] else v)
     return out
+
+
+def compact_bytes(p: int) -> int:
+    """Lb = ceil((1 + p log2 10) / 8): bitlen(10^p - 1) + 1 sign bit."""
+    return ((10 ** p - 1).bit_length() + 1 + 7) // 8
+
+
+def to_compact(mag: np.ndarray, neg: np.ndarray, p: int) -> np.ndarray:
+    """Pack sign-magnitude words into the paper's compact rows (Fig. 4):
+    Lb bytes per row, magnitude little-endian, sign in the top bit of the last
+    byte.  Pure re-packing of the generator's output (no arithmetic)."""
+    Lb = compact_bytes(p)
+    n, W = mag.shape
+    raw = np.ascontiguousarray(mag, dtype="<u4").view(np.uint8).reshape(n, 4 * W)
+    out = np.zeros((n, Lb), dtype=np.uint8)
+    k = min(Lb, 4 * W)
+    out[:, :k] = raw[:, :k]
+    out[:, Lb - 1] |= (np.asarray(neg, dtype=np.uint8) & 1) << 7
+    return out.reshape(-1)

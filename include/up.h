@@ -98,6 +98,20 @@ up_status up_column_from_host(up_ctx *ctx, const char *const *decimals, up_colum
 up_status up_column_to_host_bin(up_ctx *ctx, const up_column *col, uint32_t *mag, uint8_t *neg,
                                 void *stream);
 
+/*
+ * Compact byte-aligned column codec (the paper's cDecimal, Fig. 4):
+ * each row is Lb = up_compact_bytes(p) = ceil((1 + p log2 10)/8) bytes, the
+ * magnitude little-endian in the low 8*Lb-1 bits and the sign in the top bit
+ * of the last byte (-1.23 in DECIMAL(10,2) = {123,0,0,0,0x80}).  Rows are
+ * contiguous (row i at bytes[i*Lb]).  _host_: host buffer staged through the
+ * ctx (same lifetime rule as _host_bin); _device_: device buffer;
+ * to_host_compact synchronises the stream.  Range errors set RANGE.
+ */
+int32_t up_compact_bytes(int32_t p);
+up_status up_column_from_host_compact(up_ctx *ctx, const uint8_t *bytes, up_column *dst, void *stream);
+up_status up_column_from_device_compact(up_ctx *ctx, const uint8_t *d_bytes, up_column *dst, void *stream);
+up_status up_column_to_host_compact(up_ctx *ctx, const up_column *col, uint8_t *bytes, void *stream);
+
 /* Result type of expr over the columns (§III-B3). */
 up_status up_expr_type(up_ctx *ctx, const char *expr, const up_column *cols, int ncols,
                        int32_t *p, int32_t *s);

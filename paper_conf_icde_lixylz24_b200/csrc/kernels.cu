@@ -78,6 +78,88 @@ __global__ void __launch_bounds__(1024) k_combine(const u32 *__restrict__ parts,
     }
 }
 
+// Compact byte-aligned rows (the paper's cDecimal, P:L843-873 / Fig. 4):
+// Lb bytes per row, little-endian magnitude, the sign in the top bit of the
+// last byte.  A block stages its 256 contiguous records with 32-bit loads
+// (256*Lb is a multiple of 4), then each thread assembles its row's limbs.
+__global__ void __launch_bounds__(256) k_from_compact(const uint8_t *__restrict__ bytes, int Lb, long long n,
+                                                      const u32 *__restrict__ bound, int L, u32 *__restrict__ out,
+                                                      long long ld, u32 *flags) {
+    extern __shared__ u32 stage[];
+    const uint8_t *sb = reinterpret_cast<const uint8_t *>(stage);
+    u32 fl = 0;
+    for (long long base = (long long)blockIdx.x * 256; base < n; base += (long long)gridDim.x * 256) {
+        const long long rows = n - base < 256 ? n - base : 256;
+        const long long nbytes = rows * Lb;
+        const uint8_t *src = bytes + base * Lb;
+        __syncthreads();
+        if ((reinterpret_cast<uintptr_t>(src) & 3) == 0) {
+            const u32 *src4 = reinterpret_cast<const u32 *>(src);
+            for (long long w = threadIdx.x; w < nbytes / 4; w += blockDim.x) stage[w] = __ldcs(src4 + w);
+            for (long long b = (nbytes / 4) * 4 + threadIdx.x; b < nbytes; b += blockDim.x)
+                reinterpret_cast<uint8_t *>(stage)[b] = src[b];
+        } else {
+            for (long long b = threadIdx.x; b < nbytes; b += blockDim.x) reinterpret_cast<uint8_t *>(stage)[b] = src[b];
+        }
+        __syncthreads();
+        if (threadIdx.x < rows) {
+            const uint8_t *rb = sb + threadIdx.x * Lb;
+            const u32 ng = rb[Lb - 1] >> 7;
+            const u32 mask = 0u - ng;
+            // range: |m| < 10^p, compared limb-wise from the top
+            int cmp = 0;
+            for (int j = L - 1; j >= 0 && cmp == 0; --j) {
+                u32 m = 0;
+                for (int b = 0; b < 4; ++b) {
+                    const int k = 4 * j + b;
+                    u32 v = k < Lb ? rb[k] : 0u;
+                    if (k == Lb - 1) v &= 0x7Fu;
+                    m |= v << (8 * b);
+                }
+                if (m != bound[j]) cmp = m < bound[j] ? -1 : 1;
+            }
+            if (cmp >= 0) fl |= up::F_RANGE;
+            u64 carry = ng;
+            const long long i = base + threadIdx.x;
+            for (int j = 0; j < L; ++j) {
+                u32 m = 0;
+                for (int b = 0; b < 4; ++b) {
+                    const int k = 4 * j + b;
+                    u32 v = k < Lb ? rb[k] : 0u;
+                    if (k == Lb - 1) v &= 0x7Fu;
+                    m |= v << (8 * b);
+                }
+                const u64 t = (u64)(m ^ mask) + carry;
+                out[(long long)j * ld + i] = (u32)t;
+                carry = t >> 32;
+            }
+        }
+    }
+    if (fl) atomicOr(flags, fl);
+}
+
+// L two's-complement planes -> compact rows (Lb bytes, sign in the top bit)
+__global__ void __launch_bounds__(256) k_to_compact(const u32 *__restrict__ planes, int L, long long ld, long long n,
+                                                    uint8_t *__restrict__ bytes, int Lb) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const u32 ng = planes[(long long)(L - 1) * ld + i] >> 31;
+        const u32 mask = 0u - ng;
+        u64 carry = ng;
+        uint8_t *rb = bytes + i * Lb;
+        for (int j = 0; j < L; ++j) {
+            const u64 t = (u64)(planes[(long long)j * ld + i] ^ mask) + carry;
+            carry = t >> 32;
+            const u32 m = (u32)t;
+            for (int b = 0; b < 4; ++b) {
+                const int k = 4 * j + b;
+                if (k < Lb) rb[k] = (uint8_t)(m >> (8 * b));
+            }
+        }
+        rb[Lb - 1] = (uint8_t)((rb[Lb - 1] & 0x7Fu) | (ng << 7));
+    }
+}
+
 int grid_for(long long n, int threads) {
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
@@ -100,6 +182,28 @@ cudaError_t upk_launch_from_bin(const uint32_t *mag, int W, const uint8_t *neg, 
 cudaError_t upk_launch_to_bin(const uint32_t *planes, int L, long long ld, long long n, uint32_t *mag, uint8_t *neg,
                               cudaStream_t st) {
     k_to_bin<<<grid_for(n, 256), 256, 0, st>>>(planes, L, ld, n, mag, neg);
+    return cudaGetLastError();
+}
+
+cudaError_t upk_launch_from_compact(const uint8_t *bytes, int Lb, long long n, const uint32_t *bound, int L,
+                                   uint32_t *out, long long ld, uint32_t *flags, cudaStream_t st) {
+    const size_t smem = (size_t)256 * Lb + 16;
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(k_from_compact, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    long long want = (n + 255) / 256, cap = (long long)sms * 8;
+    k_from_compact<<<(int)(want < 1 ? 1 : (want < cap ? want : cap)), 256, smem, st>>>(bytes, Lb, n, bound, L, out, ld,
+                                                                                  flags);
+    return cudaGetLastError();
+}
+
+cudaError_t upk_launch_to_compact(const uint32_t *planes, int L, long long ld, long long n, uint8_t *bytes, int Lb,
+                                 cudaStream_t st) {
+    k_to_compact<<<grid_for(n, 256), 256, 0, st>>>(planes, L, ld, n, bytes, Lb);
     return cudaGetLastError();
 }
 

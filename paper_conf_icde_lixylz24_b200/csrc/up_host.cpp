@@ -37,6 +37,10 @@ cudaError_t upk_launch_from_bin(const uint32_t *mag, int W, const uint8_t *neg, 
 cudaError_t upk_launch_to_bin(const uint32_t *planes, int L, long long ld, long long n, uint32_t *mag, uint8_t *neg,
                               cudaStream_t st);
 cudaError_t upk_launch_combine(const uint32_t *partials, int nranks, int la, uint32_t *out, cudaStream_t st);
+cudaError_t upk_launch_from_compact(const uint8_t *bytes, int Lb, long long n, const uint32_t *bound, int L,
+                                   uint32_t *out, long long ld, uint32_t *flags, cudaStream_t st);
+cudaError_t upk_launch_to_compact(const uint32_t *planes, int L, long long ld, long long n, uint8_t *bytes, int Lb,
+                                 cudaStream_t st);
 }
 
 namespace {
@@ -478,6 +482,56 @@ up_status up_column_from_host(up_ctx *c, const char *const *decimals, up_column 
     up_status s = up_column_from_host_bin(c, mag.data(), L, neg.data(), dst, stream);
     if (s) return s;
     CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream));   // host temporaries die here
+    return UP_OK;
+}
+
+int32_t up_compact_bytes(int32_t p) {
+    // Lb = ceil((1 + p log2 10) / 8), exactly: bitlen(10^p - 1) + 1 sign bit, in bytes
+    if (p < 1) return 1;
+    HBig m = HBig::sub(HBig::pow10(p), HBig(1));
+    return (m.bitlen() + 1 + 7) / 8;
+}
+
+up_status up_column_from_device_compact(up_ctx *c, const uint8_t *d_bytes, up_column *dst, void *stream) {
+    if (!c) return fail(UP_E_INVAL, "null ctx");
+    if (up_status s = check_column(dst, "dst")) return s;
+    if (dst->n == 0) return UP_OK;
+    std::lock_guard<std::mutex> g(c->mu);
+    const uint32_t *bound = nullptr;
+    if (up_status s = pow10_device(c, dst->p, &bound)) return s;
+    CUDA_TRY(upk_launch_from_compact(d_bytes, up_compact_bytes(dst->p), dst->n, bound, dst->limbs, dst->data, dst->ld,
+                                     c->d_flags, (cudaStream_t)stream));
+    c->launches++;
+    return UP_OK;
+}
+
+up_status up_column_from_host_compact(up_ctx *c, const uint8_t *bytes, up_column *dst, void *stream) {
+    if (!c || !bytes) return fail(UP_E_INVAL, "null argument");
+    if (up_status s = check_column(dst, "dst")) return s;
+    if (dst->n == 0) return UP_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    const size_t nb = (size_t)up_compact_bytes(dst->p) * (size_t)dst->n;
+    {
+        std::lock_guard<std::mutex> g(c->mu);
+        if (up_status s = ensure_stage(c, nb, st)) return s;
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage, bytes, nb, cudaMemcpyHostToDevice, st));
+    }
+    return up_column_from_device_compact(c, (const uint8_t *)c->d_stage, dst, stream);
+}
+
+up_status up_column_to_host_compact(up_ctx *c, const up_column *col, uint8_t *bytes, void *stream) {
+    if (!c || !bytes) return fail(UP_E_INVAL, "null argument");
+    if (up_status s = check_column(col, "col")) return s;
+    if (col->n == 0) return UP_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    const int Lb = up_compact_bytes(col->p);
+    const size_t nb = (size_t)Lb * (size_t)col->n;
+    std::lock_guard<std::mutex> g(c->mu);
+    if (up_status s = ensure_stage(c, nb, st)) return s;
+    CUDA_TRY(upk_launch_to_compact(col->data, col->limbs, col->ld, col->n, (uint8_t *)c->d_stage, Lb, st));
+    c->launches++;
+    CUDA_TRY(cudaMemcpyAsync(bytes, c->d_stage, nb, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
     return UP_OK;
 }
 

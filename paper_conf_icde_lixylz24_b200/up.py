@@ -37,7 +37,8 @@ EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_l
            "up_column_to_host_bin", "up_expr_type", "up_eval_expr", "up_sum_type", "up_sum_expr",
            "up_sum", "up_sum_combine", "up_modexp", "up_modexp_sum_type", "up_modexp_sum",
            "up_sin_taylor", "up_sin_taylor_sum", "up_check", "up_format_decimal", "up_launch_count",
-           "up_jit_ms", "up_gen_source", "up_nvrtc_compile", "up_gen_modexp_source", "up_jit_prewarm", "up_gen_sin_source"]
+           "up_jit_ms", "up_gen_source", "up_nvrtc_compile", "up_gen_modexp_source", "up_jit_prewarm", "up_gen_sin_source", "up_compact_bytes",
+           "up_column_from_host_compact", "up_column_from_device_compact", "up_column_to_host_compact"]
 
 
 def lib():
@@ -80,6 +81,10 @@ def lib():
     L.up_gen_source.argtypes = [c.c_char_p, c.c_char_p, PC, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
     L.up_nvrtc_compile.argtypes = [c.c_char_p, c.c_char_p, c.c_char_p, c.c_size_t]
     L.up_jit_prewarm.argtypes = [c.c_char_p]
+    L.up_compact_bytes.argtypes = [c.c_int32]; L.up_compact_bytes.restype = c.c_int32
+    L.up_column_from_host_compact.argtypes = [P, P, PC, P]
+    L.up_column_from_device_compact.argtypes = [P, P, PC, P]
+    L.up_column_to_host_compact.argtypes = [P, PC, P, P]
     L.up_gen_sin_source.argtypes = [c.c_int32, c.c_int32, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
     L.up_gen_modexp_source.argtypes = [c.c_char_p, c.c_char_p, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
     _lib = L
@@ -93,6 +98,10 @@ def _chk(code: int):
 
 def limbs(p: int) -> int:
     return lib().up_limbs(p)
+
+
+def compact_bytes(p: int) -> int:
+    return lib().up_compact_bytes(p)
 
 
 def ld_for(n: int) -> int:
@@ -218,6 +227,30 @@ class Context:
                                              d_neg.data_ptr() if d_neg is not None else None,
                                              ctypes.byref(d), _stream_ptr(stream)))
         return col
+
+    def column_from_compact(self, p: int, s: int, data, n: Optional[int] = None, stream=None,
+                            out: Optional[Column] = None):
+        """Compact rows: numpy uint8 / pinned torch uint8 (host) or a CUDA uint8 tensor."""
+        import numpy as np
+        Lb = compact_bytes(p)
+        if isinstance(data, np.ndarray):
+            n = data.size // Lb if n is None else n
+            ptr, dev = data.ctypes.data, False
+        else:
+            n = data.numel() // Lb if n is None else n
+            ptr, dev = data.data_ptr(), data.is_cuda
+        col = out if out is not None else Column(p, s, n)
+        d = col.desc()
+        fn = lib().up_column_from_device_compact if dev else lib().up_column_from_host_compact
+        _chk(fn(self.h, ptr, ctypes.byref(d), _stream_ptr(stream)))
+        return col
+
+    def column_to_compact(self, col: Column, stream=None):
+        import numpy as np
+        out = np.zeros(max(1, col.n * compact_bytes(col.p)), dtype=np.uint8)
+        d = col.desc()
+        _chk(lib().up_column_to_host_compact(self.h, ctypes.byref(d), out.ctypes.data, _stream_ptr(stream)))
+        return out[: col.n * compact_bytes(col.p)]
 
     def column_from_strings(self, p: int, s: int, values: Sequence[str], stream=None):
         col = Column(p, s, len(values))
