@@ -196,6 +196,10 @@ double up_jit_ms(up_ctx *ctx);
 up_status up_gen_source(const char *variant, const char *expr, const up_column *cols, int ncols,
                         int64_t n_global, char *buf, size_t len);
 up_status up_nvrtc_compile(const char *src, const char *cubin_path, char *log, size_t len);
+/* The expression after the optimiser (alignment scheduling + constant
+ * pre-calculation; value-preserving, root kept at the
+ * unoptimised type), as canonical text "tree : (p,s)" (no GPU needed). */
+up_status up_expr_optimized(const char *expr, const up_column *cols, int ncols, char *buf, size_t len);
 /* Compile a generated source into the on-disk cubin cache ($UP_JIT_CACHE,
  * else <dir of libup.so>/_jitcache) so a GPU process loads it without NVRTC. */
 up_status up_jit_prewarm(const char *src);

@@ -72,6 +72,10 @@ struct Emitter {
             o << "    const u32 " << t << "[" << n->L << "] = " << limbs_init(n->lit.twos(n->L, false)) << ";\n";
             return t;
         }
+        case Op::Cast: {   // exact upward re-typing (optimiser output)
+            std::string a = emit(n->l.get());
+            return aligned(a, n->l->L, n->s - n->l->s, n->L);
+        }
         case Op::Neg: {
             std::string a = emit(n->l.get());
             std::string t = fresh("t");

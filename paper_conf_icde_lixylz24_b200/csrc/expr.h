@@ -9,7 +9,7 @@
 
 namespace uph {
 
-enum class Op { Col, Lit, Add, Sub, Mul, Div, Mod, Neg };
+enum class Op { Col, Lit, Add, Sub, Mul, Div, Mod, Neg, Cast };
 
 struct Node {
     Op op = Op::Lit;
@@ -37,6 +37,15 @@ int sum_precision(int p, long long n_global);
 
 // canonical text of a typed tree (cache key component)
 std::string canonical(const Node *n);
+
+// Expression optimiser (§III-D): alignment scheduling (- as
+// unary negation, + collapsed to n-ary, terms ordered by scale, rebuilt as a
+// binary tree) and constant pre-calculation / shortcuts (constants folded per
+// level, +a / 0+a / 1*a removed).  Value-preserving: +, -, * are exact, and
+// the operands of / and % keep their original types (Cast), so every row's
+// value -- including every truncation and every flag -- is unchanged; the
+// root is cast back to the unoptimised (p,s) (reading Q12).
+std::unique_ptr<Node> optimize(const Node *typed_root, const std::vector<ColType> &cols);
 
 bool uses_divmod(const Node *n);
 int max_limbs(const Node *n);

@@ -335,12 +335,16 @@ up_status expr_kernel(up_ctx *c, const char *expr, const up_column *cols, int nc
     o.LA = LA;
     GenInfo info;
     std::string src;
+    // expression optimiser (alignment scheduling + constant pre-calculation),
+    // value-preserving; the kernel is generated from the optimised tree
+    std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(t.root.get(), t.types);
+    const Node *gen_root = opt_root ? opt_root.get() : t.root.get();
     // wide SUM regime: warp per row, linear decomposition into summed terms
-    if (sum && max_limbs(t.root.get()) >= kWideMinLimbs && LA <= 512 && !getenv("UP_NO_WIDE"))
-        src = gen_wide_sum_kernel(t.root.get(), t.types, LA, info);
+    if (sum && max_limbs(gen_root) >= kWideMinLimbs && LA <= 512 && !getenv("UP_NO_WIDE"))
+        src = gen_wide_sum_kernel(gen_root, t.types, LA, info);
     if (src.empty()) {
         info = GenInfo();
-        src = gen_expr_kernel(t.root.get(), t.types, o, info);
+        src = gen_expr_kernel(gen_root, t.types, o, info);
     }
     if (sum && info.ws_slots > kWsSlots) return fail(UP_E_UNSUPPORTED, "SUM too wide (%d slots)", info.ws_slots);
     JitKernel *k = nullptr;
@@ -681,9 +685,11 @@ up_status up_gen_source(const char *variant, const char *expr, const up_column *
     o.LA = o.sum ? limbs_for_precision(sum_precision(t.root->p, N)) : 0;
     GenInfo info;
     std::string src;
-    if (o.sum && max_limbs(t.root.get()) >= kWideMinLimbs && o.LA <= 512 && !getenv("UP_NO_WIDE"))
-        src = gen_wide_sum_kernel(t.root.get(), t.types, o.LA, info);
-    if (src.empty()) src = gen_expr_kernel(t.root.get(), t.types, o, info);
+    std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(t.root.get(), t.types);
+    const Node *gen_root = opt_root ? opt_root.get() : t.root.get();
+    if (o.sum && max_limbs(gen_root) >= kWideMinLimbs && o.LA <= 512 && !getenv("UP_NO_WIDE"))
+        src = gen_wide_sum_kernel(gen_root, t.types, o.LA, info);
+    if (src.empty()) src = gen_expr_kernel(gen_root, t.types, o, info);
     if (src.size() + 1 > len) return fail(UP_E_NOMEM, "need %zu bytes", src.size() + 1);
     memcpy(buf, src.c_str(), src.size() + 1);
     return UP_OK;
@@ -712,6 +718,17 @@ up_status up_nvrtc_compile(const char *src, const char *cubin_path, char *log, s
         std::ofstream(cubin_path, std::ios::binary).write(cubin.data(), (std::streamsize)cs);
     }
     nvrtcDestroyProgram(&prog);
+    return UP_OK;
+}
+
+// Canonical text of the optimised tree (alignment scheduling + constant folding)
+up_status up_expr_optimized(const char *expr, const up_column *cols, int ncols, char *buf, size_t len) {
+    Typed t;
+    if (up_status s = type_expr(expr, cols, ncols, t)) return s;
+    auto o = optimize(t.root.get(), t.types);
+    std::string txt = canonical(o.get()) + " : (" + std::to_string(o->p) + "," + std::to_string(o->s) + ")";
+    if (txt.size() + 1 > len) return fail(UP_E_NOMEM, "buffer too small");
+    memcpy(buf, txt.c_str(), txt.size() + 1);
     return UP_OK;
 }
 
