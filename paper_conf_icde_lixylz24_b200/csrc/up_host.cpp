@@ -305,6 +305,8 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     k += expr;
     for (int i = 0; i < ncols; ++i) k += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
     k += "|" + std::to_string(extra);
+    if (getenv("UP_NO_OPT")) k += "|noopt";
+    if (getenv("UP_NO_WIDE")) k += "|nowide";
     return k;
 }
 
