@@ -133,6 +133,8 @@ struct up_ctx {
     uint32_t *d_flags = nullptr;
     void *d_stage = nullptr;
     size_t stage_bytes = 0;
+    void *d_scratch = nullptr;   // kernel scratch (sin_P running sums), grown on demand
+    size_t scratch_bytes = 0;
     std::map<int, uint32_t *> pow10_dev;  // 10^p magnitude in up_limbs(p) limbs
     std::unordered_map<std::string, std::unique_ptr<JitKernel>> by_src;
     std::unordered_map<std::string, JitKernel *> by_key;
@@ -417,6 +419,7 @@ up_status up_ctx_destroy(up_ctx *c) {
     cudaFree(c->d_ticket);
     cudaFree(c->d_flags);
     if (c->d_stage) cudaFree(c->d_stage);
+    if (c->d_scratch) cudaFree(c->d_scratch);
     delete c;
     return UP_OK;
 }
@@ -777,4 +780,18 @@ std::mutex &up_internal_mutex(up_ctx *c) { return c->mu; }
 unsigned long long *up_internal_ws(up_ctx *c) { return c->d_ws; }
 uint32_t *up_internal_ticket(up_ctx *c) { return c->d_ticket; }
 uint32_t *up_internal_flags(up_ctx *c) { return c->d_flags; }
+int up_internal_num_sms(up_ctx *c) { return c->num_sms; }
+up_status up_internal_scratch(up_ctx *c, size_t bytes, void **out) {
+    if (bytes > c->scratch_bytes) {
+        if (c->d_scratch) {
+            CUDA_TRY(cudaDeviceSynchronize());
+            CUDA_TRY(cudaFree(c->d_scratch));
+            c->d_scratch = nullptr;
+        }
+        CUDA_TRY(cudaMalloc(&c->d_scratch, bytes));
+        c->scratch_bytes = bytes;
+    }
+    *out = c->d_scratch;
+    return UP_OK;
+}
 up_status up_internal_fail(up_status st, const std::string &msg) { return fail(st, "%s", msg.c_str()); }

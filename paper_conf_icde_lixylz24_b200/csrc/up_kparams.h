@@ -14,4 +14,6 @@ typedef struct {
     unsigned int *ticket;                  /* sum: last-block ticket (zeroed) */
     unsigned int *result;                  /* sum: LA-limb two's-complement partial */
     unsigned int *flags;                   /* sticky error flags (F_*) */
+    unsigned int *scratch;                 /* per-thread global scratch (sin_P running sums) */
+    long long scratch_stride;              /* elements between consecutive words of one thread */
 } up_kparams;
