@@ -71,3 +71,23 @@ def test_sin_odd_symmetry_on_gpu():
             assert u == v
         else:
             assert u == ("-" + v if not v.startswith("-") else v[1:])
+
+
+@pytest.mark.parametrize("P,n", [(20, 200), (300, 50), (1400, 6)])
+@pytest.mark.parametrize("pst", [(9, 8), (5, 2), (1, 0)])
+def test_sin_shared_memory_variant(P, n, pst, monkeypatch):
+    """The t-in-shared-memory / S-in-scratch kernel (default for 128 < W <= 200
+    limbs, forced here with UP_SIN_SMEM) against the oracle, incl. scales whose
+    constant shift is a left shift (s = 2) or absent (s = 0)."""
+    monkeypatch.setenv("UP_SIN_SMEM", "1")
+    p, s = pst
+    mag, neg = synth.uniform_decimal(n, p, 5, 4)
+    c = G.ctx()
+    x = c.column_from_host_bin(p, s, mag, neg)
+    out = c.sin_taylor(x, P)
+    c.check()
+    assert c.column_to_strings(out) == oracle.sin_rows(oracle.Column(p, s, mag, neg), P)
+    from paper_conf_icde_lixylz24_b200 import up
+    res = c.sin_taylor_sum(x, P)
+    c.check()
+    assert up.result_to_string(res, P) == oracle.sin_sum(oracle.Column(p, s, mag, neg), P, threads=8)
