@@ -166,7 +166,8 @@ up_status up_modexp_sum(up_ctx *ctx, const up_column *base, const char *exponent
 
 /*
  * Fixed-point Taylor sine sin_P(x) per row (row a9, from
- * Query 5 P:L2197-2249): x DECIMAL(p,s) with s <= 9, p - s <= 1 (|x| < 10),
+ * Query 5 P:L2197-2249): x DECIMAL(p,s) with p <= 9, p - s <= 1 (|x| < 10, else
+ * UP_E_UNSUPPORTED), s <= P,
  * t_1 = |m_x| 10^(P-s), t_{k+1} = floor(t_k m_x^2 / (10^(2s) (2k)(2k+1))),
  * result sign(m_x) * sum_k (-1)^(k-1) t_k, type DECIMAL(P+1, P).
  * up_sin_taylor: out caller-allocated DECIMAL(P+1,P).
