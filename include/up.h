@@ -201,6 +201,8 @@ up_status up_nvrtc_compile(const char *src, const char *cubin_path, char *log, s
  * pre-calculation; value-preserving, root kept at the
  * unoptimised type), as canonical text "tree : (p,s)" (no GPU needed). */
 up_status up_expr_optimized(const char *expr, const up_column *cols, int ncols, char *buf, size_t len);
+/* Generated row-contraction source for SUM(c1*c2) with La x Lb limbs (sign +1/-1). */
+up_status up_gen_contract_source(int32_t La, int32_t Lb, int32_t LA, int sign, char *buf, size_t len);
 /* Compile a generated source into the on-disk cubin cache ($UP_JIT_CACHE,
  * else <dir of libup.so>/_jitcache) so a GPU process loads it without NVRTC. */
 up_status up_jit_prewarm(const char *src);

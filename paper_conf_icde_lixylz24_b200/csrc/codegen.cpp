@@ -431,4 +431,186 @@ std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &co
     k << "}\n";
     return k.str();
 }
+
+// ---------------------------------------------------------------------------
+// Row contraction for SUM of a column product (cfg3's c1*c2): over all rows,
+// sum a*b = sum_k 2^(32k) sum_{i+j=k} (sum_rows A_i B_j)  -  sign corrections,
+// with A, B the raw two's-complement limbs read as unsigned (a = A - s_a 2^(32 La)):
+//   sum ab = sum AB - 2^(32 La) sum s_a B - 2^(32 Lb) sum s_b A + 2^(32(La+Lb)) sum s_a s_b.
+// Each warp owns K consecutive product columns and keeps exact 96-bit
+// carry-save column sums across all its rows (one row per lane): per a-limb
+// one load of A_i and one of the sliding B window, K IMAD.WIDE products, no
+// per-row carry propagation and no per-row sign handling.  The last block
+// normalises pos - neg into LA limbs (negated for a '-' term) at P.result.
+std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int col_b, GenInfo &info) {
+    const int NK = La + Lb + 1;                 // columns 0 .. La+Lb (the last for s_a s_b)
+    const int K = (NK + 7) / 8 <= 16 ? 8 : 16;  // keep a block <= 16 warps (registers per thread)
+    const int CR = (NK + K - 1) / K;            // column ranges = warps per block
+    const int NSL = NK + 3;                     // slot columns (carries of the top column)
+    if (CR > 32) return "";
+    info.threads = CR * 32;
+    info.rows_per_block = 32;
+    info.ws_slots = 2 * NSL;
+    info.dyn_smem = 0;
+    std::ostringstream k;
+    k << "// generated by libup: row contraction SUM(c" << col_a + 1 << "*c" << col_b + 1 << ") La=" << La << " Lb=" << Lb
+      << " K=" << K << " ranges=" << CR << "\n";
+    k << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
+    k << "extern \"C\" __global__ void __launch_bounds__(" << CR * 32 << ") upk(const up_kparams P) {\n";
+    k << "    constexpr int LA_ = " << La << ", LB_ = " << Lb << ", K = " << K << ", NSL = " << NSL << ";\n";
+    k << "    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n";
+    k << "    const int k0 = warp * K;\n";
+    k << "    const u32 *A = P.col[" << col_a << "], *B = P.col[" << col_b << "];\n";
+    k << "    const long long lda = P.ld[" << col_a << "], ldb = P.ld[" << col_b << "];\n";
+    k << "    u64 lo[K], cor[K]; u32 hi[K]; u64 ss = 0;\n";
+    k << "#pragma unroll\n    for (int m = 0; m < K; ++m) { lo[m] = 0ull; hi[m] = 0u; cor[m] = 0ull; }\n";
+    k << "    const int ilo = k0 - (LB_ - 1) > 0 ? k0 - (LB_ - 1) : 0;\n";
+    k << "    const int ihi = k0 + K - 1 < LA_ - 1 ? k0 + K - 1 : LA_ - 1;\n";
+    k << "    const long long n = P.n;\n";
+    k << "    for (long long r0 = (long long)blockIdx.x * 32; r0 < n; r0 += (long long)gridDim.x * 32) {\n";
+    k << "        const long long row = r0 + lane;\n";
+    k << "        if (row < n) {\n";
+    // window w[m] = B_{k0 + m - i}
+    k << "            u32 w[K];\n";
+    k << "#pragma unroll\n            for (int m = 0; m < K; ++m) { const int j = k0 + m - ilo; w[m] = (j >= 0 && j < LB_) ? __ldg(B + (long long)j * ldb + row) : 0u; }\n";
+    k << "            for (int i = ilo; i <= ihi; ++i) {\n";
+    k << "                const u32 ai = __ldg(A + (long long)i * lda + row);\n";
+    k << "#pragma unroll\n                for (int m = 0; m < K; ++m) {\n";
+    k << "                    const u64 p = (u64)ai * w[m];\n";
+    k << "                    const u64 s = lo[m] + p;\n";
+    k << "                    hi[m] += s < p ? 1u : 0u;\n";
+    k << "                    lo[m] = s;\n";
+    k << "                }\n";
+    k << "                // slide the window: w[m] <- B_{k0 + m - (i+1)}\n";
+    k << "#pragma unroll\n                for (int m = K - 1; m > 0; --m) w[m] = w[m - 1];\n";
+    k << "                { const int j = k0 - i - 1; w[0] = (j >= 0 && j < LB_) ? __ldg(B + (long long)j * ldb + row) : 0u; }\n";
+    k << "            }\n";
+    // sign corrections
+    k << "            const u32 sa = __ldg(A + (long long)(LA_ - 1) * lda + row) >> 31;\n";
+    k << "            const u32 sb = __ldg(B + (long long)(LB_ - 1) * ldb + row) >> 31;\n";
+    k << "            if (sa) {\n#pragma unroll\n              for (int m = 0; m < K; ++m) { const int j = k0 + m - LA_; if (j >= 0 && j < LB_) cor[m] += __ldg(B + (long long)j * ldb + row); } }\n";
+    k << "            if (sb) {\n#pragma unroll\n              for (int m = 0; m < K; ++m) { const int j = k0 + m - LB_; if (j >= 0 && j < LA_) cor[m] += __ldg(A + (long long)j * lda + row); } }\n";
+    k << "            ss += sa & sb;\n";
+    k << "        }\n";
+    k << "    }\n";
+    // warp reduce
+    k << "#pragma unroll\n    for (int m = 0; m < K; ++m) {\n";
+    k << "#pragma unroll\n        for (int o = 16; o > 0; o >>= 1) {\n";
+    k << "            const u64 l2 = __shfl_down_sync(0xFFFFFFFFu, lo[m], o); const u32 h2 = __shfl_down_sync(0xFFFFFFFFu, hi[m], o);\n";
+    k << "            const u64 s = lo[m] + l2; hi[m] += h2 + (s < l2 ? 1u : 0u); lo[m] = s;\n";
+    k << "            cor[m] += __shfl_down_sync(0xFFFFFFFFu, cor[m], o);\n";
+    k << "        }\n    }\n";
+    k << "#pragma unroll\n    for (int o = 16; o > 0; o >>= 1) ss += __shfl_down_sync(0xFFFFFFFFu, ss, o);\n";
+    k << "    u64 *pos = P.ws, *neg = P.ws + NSL;\n";
+    k << "    if (lane == 0) {\n";
+    k << "#pragma unroll\n        for (int m = 0; m < K; ++m) {\n";
+    k << "            const int col = k0 + m;\n";
+    k << "            if (col + 2 < NSL) {\n";
+    k << "                if ((u32)lo[m]) atomicAdd(&pos[col], (u64)(u32)lo[m]);\n";
+    k << "                if (lo[m] >> 32) atomicAdd(&pos[col + 1], lo[m] >> 32);\n";
+    k << "                if (hi[m]) atomicAdd(&pos[col + 2], (u64)hi[m]);\n";
+    k << "                if ((u32)cor[m]) atomicAdd(&neg[col], (u64)(u32)cor[m]);\n";
+    k << "                if (cor[m] >> 32) atomicAdd(&neg[col + 1], cor[m] >> 32);\n";
+    k << "            }\n        }\n";
+    k << "        if (warp == 0 && ss) atomicAdd(&pos[LA_ + LB_], ss);\n";
+    k << "    }\n";
+    // last block: normalise pos - neg (sign) into LA limbs
+    k << "    __threadfence();\n    __syncthreads();\n";
+    k << "    __shared__ u32 s_last;\n";
+    k << "    if (threadIdx.x == 0) s_last = (atomicAdd(P.ticket, 1u) == gridDim.x - 1) ? 1u : 0u;\n";
+    k << "    __syncthreads();\n    if (!s_last) return;\n    __threadfence();\n";
+    k << "    __shared__ u64 sp[NSL], sn[NSL];\n";
+    k << "    for (int i = threadIdx.x; i < NSL; i += blockDim.x) { sp[i] = atomicExch(&pos[i], 0ull); sn[i] = atomicExch(&neg[i], 0ull); }\n";
+    k << "    __syncthreads();\n";
+    k << "    if (threadIdx.x == 0) {\n";
+    k << "        *P.ticket = 0u;\n";
+    k << "        u64 cp = 0, cn = 0; u32 borrow = 0, cneg = " << (sign < 0 ? 1 : 0) << "u;\n";
+    k << "        for (int j = 0; j < " << LA << "; ++j) {\n";
+    k << "            u64 tp = cp, tn = cn;\n";
+    k << "            if (j < NSL) { tp += (u32)sp[j]; tn += (u32)sn[j]; }\n";
+    k << "            if (j >= 1 && j - 1 < NSL) { tp += sp[j - 1] >> 32; tn += sn[j - 1] >> 32; }\n";
+    k << "            cp = tp >> 32; cn = tn >> 32;\n";
+    k << "            const u64 d = (u64)(u32)tp - (u32)tn - borrow;\n";
+    k << "            borrow = (u32)(d >> 63);\n";
+    if (sign < 0) {
+        k << "            const u64 ng = (u64)(~(u32)d) + cneg; cneg = (u32)(ng >> 32);\n";
+        k << "            P.result[j] = (u32)ng;\n";
+    } else {
+        k << "            P.result[j] = (u32)d;\n";
+    }
+    k << "        }\n    }\n";
+    k << "}\n";
+    return k.str();
+}
+
+namespace {
+void flatten_any(const Node *n, int sign, std::vector<std::pair<int, const Node *>> &out) {
+    switch (n->op) {
+    case Op::Add: flatten_any(n->l.get(), sign, out); flatten_any(n->r.get(), sign, out); return;
+    case Op::Sub: flatten_any(n->l.get(), sign, out); flatten_any(n->r.get(), -sign, out); return;
+    case Op::Neg: flatten_any(n->l.get(), -sign, out); return;
+    default: out.push_back({sign, n}); return;
+    }
+}
+std::unique_ptr<Node> clone_node(const Node *n) {
+    auto c = std::make_unique<Node>();
+    c->op = n->op; c->col = n->col; c->lit = n->lit; c->p = n->p; c->s = n->s; c->L = n->L;
+    if (n->l) c->l = clone_node(n->l.get());
+    if (n->r) c->r = clone_node(n->r.get());
+    return c;
+}
+}  // namespace
+
+// SUM(root) = sum of SUM(+-ci*cj) over the top-level column-product terms at
+// the output scale (row contraction kernels) + SUM(rest) with the rest cast to
+// the output scale (fused per-thread kernel).  Exact: SUM is linear and every
+// term is an exact part of the row value.  Products below another scale, or
+// too small to be compute-bound, stay in the rest.
+bool split_sum_terms(const Node *root, const std::vector<ColType> &cols, int min_products,
+                     std::vector<SplitTerm> &prods, std::unique_ptr<Node> &rest) {
+    const Node *body = root->op == Op::Cast ? root->l.get() : root;
+    const int s_out = root->s;
+    std::vector<std::pair<int, const Node *>> terms;
+    flatten_any(body, 1, terms);
+    std::vector<std::pair<int, const Node *>> others;
+    for (auto &t : terms) {
+        const Node *n = t.second;
+        if (n->op == Op::Mul && n->l->op == Op::Col && n->r->op == Op::Col && n->s == s_out &&
+            cols[(size_t)n->l->col].limbs * cols[(size_t)n->r->col].limbs >= min_products)
+            prods.push_back({t.first, n->l->col, n->r->col});
+        else
+            others.push_back(t);
+    }
+    if (prods.empty()) return false;
+    rest.reset();
+    if (!others.empty()) {
+        std::unique_ptr<Node> acc;
+        bool acc_neg = false;
+        for (auto &t : others) {
+            auto c = clone_node(t.second);
+            const bool ng = t.first < 0;
+            if (!acc) { acc = std::move(c); acc_neg = ng; continue; }
+            auto m = std::make_unique<Node>();
+            if (acc_neg && !ng) { m->op = Op::Sub; m->l = std::move(c); m->r = std::move(acc); acc_neg = false; }
+            else { m->op = acc_neg == ng ? Op::Add : Op::Sub; m->l = std::move(acc); m->r = std::move(c); }
+            acc = std::move(m);
+        }
+        if (acc_neg) { auto m = std::make_unique<Node>(); m->op = Op::Neg; m->l = std::move(acc); acc = std::move(m); }
+        std::string err;
+        type_tree(acc.get(), cols, err);
+        if (!err.empty() || acc->s > s_out) return false;
+        if (acc->s < s_out) {
+            auto cst = std::make_unique<Node>();
+            cst->op = Op::Cast;
+            cst->p = acc->p + (s_out - acc->s);
+            cst->s = s_out;
+            cst->L = limbs_for_precision(cst->p);
+            cst->l = std::move(acc);
+            acc = std::move(cst);
+            type_tree(acc.get(), cols, err);
+        }
+        rest = std::move(acc);
+    }
+    return true;
+}
 }  // namespace uph

@@ -21,6 +21,13 @@ struct GenInfo {
 };
 
 std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, const GenOpts &opt, GenInfo &info);
+// row contraction of SUM(ci*cj) (see codegen.cpp)
+struct SplitTerm {
+    int sign, col_a, col_b;
+};
+std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int col_b, GenInfo &info);
+bool split_sum_terms(const Node *root, const std::vector<ColType> &cols, int min_products,
+                     std::vector<SplitTerm> &prods, std::unique_ptr<Node> &rest);
 // wide SUM regime (warp per row); "" if the expression does not fit it
 std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &cols, int LA, GenInfo &info);
 

@@ -109,6 +109,7 @@ up_status fail(up_status st, const char *fmt, ...) {
 
 constexpr int kThreads = 256;
 constexpr int kWsSlots = 1 << 16;
+constexpr int kContractMinProducts = 100;   // row contraction only for compute-bound products
 constexpr int kWideMinLimbs = 257;  // warp-per-row only beyond this (per-thread measured faster at p <= 1000)
 
 struct JitKernel {
@@ -135,6 +136,8 @@ struct up_ctx {
     size_t stage_bytes = 0;
     void *d_scratch = nullptr;   // kernel scratch (sin_P running sums), grown on demand
     size_t scratch_bytes = 0;
+    uint32_t *d_parts = nullptr; // per-term SUM partials of a split SUM
+    size_t parts_words = 0;
     std::map<int, uint32_t *> pow10_dev;  // 10^p magnitude in up_limbs(p) limbs
     std::unordered_map<std::string, std::unique_ptr<JitKernel>> by_src;
     std::unordered_map<std::string, JitKernel *> by_key;
@@ -371,6 +374,34 @@ up_status expr_kernel(up_ctx *c, const char *expr, const up_column *cols, int nc
     return UP_OK;
 }
 
+// compile (or fetch) a kernel generated by `gen` under `key`, applying its launch info
+template <class Gen>
+up_status kernel_for(up_ctx *c, const std::string &key, Gen gen, JitKernel **out) {
+    auto it = c->by_key.find(key);
+    if (it != c->by_key.end()) { *out = it->second; return UP_OK; }
+    GenInfo info;
+    std::string src = gen(info);
+    if (src.empty()) return fail(UP_E_UNSUPPORTED, "no kernel for %s", key.c_str());
+    if (info.ws_slots > kWsSlots) return fail(UP_E_UNSUPPORTED, "SUM too wide (%d slots)", info.ws_slots);
+    JitKernel *k = nullptr;
+    if (up_status s = compile(c, src, &k)) return s;
+    k->rows_per_thread = info.rows_per_thread;
+    k->ws_slots = info.ws_slots;
+    k->rows_per_block = info.rows_per_block;
+    if (info.threads != k->threads || info.dyn_smem != k->dyn_smem) {
+        k->threads = info.threads;
+        if (info.dyn_smem > 48 * 1024)
+            CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, info.dyn_smem));
+        k->dyn_smem = info.dyn_smem;
+        int nb = 0;
+        CU_TRY(drv.OccupancyMaxActiveBlocksPerMultiprocessor(&nb, k->fn, k->threads, (size_t)k->dyn_smem));
+        k->blocks_per_sm = std::max(1, nb);
+    }
+    c->by_key[key] = k;
+    *out = k;
+    return UP_OK;
+}
+
 void fill_cols(up_kparams &P, const up_column *cols, int ncols) {
     memset(&P, 0, sizeof P);
     for (int i = 0; i < ncols; ++i) {
@@ -420,6 +451,7 @@ up_status up_ctx_destroy(up_ctx *c) {
     cudaFree(c->d_flags);
     if (c->d_stage) cudaFree(c->d_stage);
     if (c->d_scratch) cudaFree(c->d_scratch);
+    if (c->d_parts) cudaFree(c->d_parts);
     delete c;
     return UP_OK;
 }
@@ -621,6 +653,60 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     Typed t;
     const long long N = n_global > 0 ? n_global : cols[0].n;
     if (N < cols[0].n) return fail(UP_E_INVAL, "n_global < local rows");
+    // Split SUM: top-level column products -> row-contraction kernels, the
+    // rest -> the fused per-thread kernel, then an exact combine (SUM is linear).
+    if (!getenv("UP_NO_SPLIT")) {
+        Typed ts;
+        if (up_status s = type_expr(expr, cols, ncols, ts)) return s;
+        const int LAs = limbs_for_precision(sum_precision(ts.root->p, N));
+        std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(ts.root.get(), ts.types);
+        const Node *base = opt_root ? opt_root.get() : ts.root.get();
+        std::vector<SplitTerm> prods;
+        std::unique_ptr<Node> rest;
+        if (LAs <= 512 && split_sum_terms(base, ts.types, kContractMinProducts, prods, rest)) {
+            const int T = (int)prods.size() + (rest ? 1 : 0);
+            const size_t need = (size_t)T * (size_t)LAs;
+            if (need > c->parts_words) {
+                if (c->d_parts) { CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream)); CUDA_TRY(cudaFree(c->d_parts)); }
+                CUDA_TRY(cudaMalloc(&c->d_parts, sizeof(uint32_t) * need * 2));
+                c->parts_words = need * 2;
+            }
+            up_kparams P;
+            fill_cols(P, cols, ncols);
+            P.ws = c->d_ws;
+            P.ticket = c->d_ticket;
+            P.flags = c->d_flags;
+            int ti = 0;
+            for (const SplitTerm &st : prods) {
+                const int La = cols[st.col_a].limbs, Lb = cols[st.col_b].limbs;
+                std::string key = "contract|" + std::to_string(La) + "|" + std::to_string(Lb) + "|" + std::to_string(LAs) +
+                                  "|" + std::to_string(st.sign) + "|" + std::to_string(st.col_a) + "|" + std::to_string(st.col_b);
+                JitKernel *kc = nullptr;
+                if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
+                        return gen_contract_kernel(La, Lb, LAs, st.sign, st.col_a, st.col_b, info); }, &kc))
+                    return s;
+                P.result = c->d_parts + (size_t)ti++ * LAs;
+                if (up_status s = launch(c, kc, P, P.n, (cudaStream_t)stream)) return s;
+            }
+            if (rest) {
+                std::string key = "rest|" + canonical(rest.get()) + "|" + std::to_string(LAs);
+                for (int i = 0; i < ncols; ++i) key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
+                JitKernel *kr = nullptr;
+                Node *rr = rest.get();
+                if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
+                        GenOpts o;
+                        o.sum = true;
+                        o.LA = LAs;
+                        return gen_expr_kernel(rr, ts.types, o, info); }, &kr))
+                    return s;
+                P.result = c->d_parts + (size_t)ti++ * LAs;
+                if (up_status s = launch(c, kr, P, P.n, (cudaStream_t)stream)) return s;
+            }
+            CUDA_TRY(upk_launch_combine(c->d_parts, T, LAs, d_partial, (cudaStream_t)stream));
+            c->launches++;
+            return UP_OK;
+        }
+    }
     if (up_status s = expr_kernel(c, expr, cols, ncols, true, N, &k, &LA, nullptr, t)) return s;
     up_kparams P;
     fill_cols(P, cols, ncols);
@@ -734,6 +820,16 @@ up_status up_expr_optimized(const char *expr, const up_column *cols, int ncols, 
     std::string txt = canonical(o.get()) + " : (" + std::to_string(o->p) + "," + std::to_string(o->s) + ")";
     if (txt.size() + 1 > len) return fail(UP_E_NOMEM, "buffer too small");
     memcpy(buf, txt.c_str(), txt.size() + 1);
+    return UP_OK;
+}
+
+// generated row-contraction source (diagnostics / prewarm)
+up_status up_gen_contract_source(int32_t La, int32_t Lb, int32_t LA, int sign, char *buf, size_t len) {
+    GenInfo info;
+    std::string src = gen_contract_kernel(La, Lb, LA, sign, 0, 1, info);
+    if (src.empty()) return fail(UP_E_UNSUPPORTED, "no contraction kernel");
+    if (src.size() + 1 > len) return fail(UP_E_NOMEM, "buffer too small");
+    memcpy(buf, src.c_str(), src.size() + 1);
     return UP_OK;
 }
 

@@ -39,7 +39,7 @@ EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_l
            "up_sin_taylor", "up_sin_taylor_sum", "up_check", "up_format_decimal", "up_launch_count",
            "up_jit_ms", "up_gen_source", "up_nvrtc_compile", "up_gen_modexp_source", "up_jit_prewarm", "up_gen_sin_source", "up_compact_bytes",
            "up_column_from_host_compact", "up_column_from_device_compact", "up_column_to_host_compact",
-           "up_expr_optimized"]
+           "up_expr_optimized", "up_gen_contract_source"]
 
 
 def lib():
@@ -84,6 +84,7 @@ def lib():
     L.up_jit_prewarm.argtypes = [c.c_char_p]
     L.up_compact_bytes.argtypes = [c.c_int32]; L.up_compact_bytes.restype = c.c_int32
     L.up_expr_optimized.argtypes = [c.c_char_p, PC, c.c_int, c.c_char_p, c.c_size_t]
+    L.up_gen_contract_source.argtypes = [c.c_int32, c.c_int32, c.c_int32, c.c_int, c.c_char_p, c.c_size_t]
     L.up_column_from_host_compact.argtypes = [P, P, PC, P]
     L.up_column_from_device_compact.argtypes = [P, P, PC, P]
     L.up_column_to_host_compact.argtypes = [P, PC, P, P]
@@ -423,6 +424,12 @@ def expr_optimized(expr: str, types: Sequence[tuple]) -> str:
         arr[i] = up_column(1, 4, p, s, limbs(p), 0, None)
     buf = ctypes.create_string_buffer(1 << 16)
     _chk(lib().up_expr_optimized(expr.encode(), arr, len(types), buf, len(buf)))
+    return buf.value.decode()
+
+
+def gen_contract_source(La: int, Lb: int, LA: int, sign: int = 1) -> str:
+    buf = ctypes.create_string_buffer(1 << 20)
+    _chk(lib().up_gen_contract_source(La, Lb, LA, sign, buf, len(buf)))
     return buf.value.decode()
 
 

@@ -77,3 +77,27 @@ def test_wide_and_per_thread_paths_agree(monkeypatch):
     narrow = up.result_to_string(c2.sum_expr("c1*c2 - c3/c4", cols2), S)
     c2.check()
     assert wide == narrow
+
+
+@pytest.mark.parametrize("expr,types,lead", [
+    ("c1*c2 - c3/c4", [(200, 50)] * 4, (3,)),
+    ("c1*c2", [(120, 30), (90, 20)], ()),
+    ("-c1*c2 + c3*c1 - c2", [(150, 10), (150, 10), (140, 10)], ()),
+    ("c1*c2 - c3/c4", [(1000, 100)] * 4, (3,)),
+])
+def test_split_sum_matches_unsplit_and_oracle(expr, types, lead, monkeypatch):
+    """Row-contraction SUM (products as carry-save column sums over rows, signs
+    by correction terms) + fused rest kernel + combine == oracle == UP_NO_SPLIT."""
+    n = 300 if types[0][0] >= 1000 else 2000
+    host = G.gen_cols(n, types, config=3, nonzero_lead_cols=lead, seed=11)
+    want, P, S = oracle.eval_sum(expr, G.to_oracle(host, types), threads=8)
+    from paper_conf_icde_lixylz24_b200 import up
+    c = up.Context(0)
+    cols = [c.column_from_host_bin(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
+    got = up.result_to_string(c.sum_expr(expr, cols), S)
+    c.check()
+    assert got == want
+    monkeypatch.setenv("UP_NO_SPLIT", "1")
+    c2 = up.Context(0)
+    cols2 = [c2.column_from_host_bin(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
+    assert up.result_to_string(c2.sum_expr(expr, cols2), S) == want
