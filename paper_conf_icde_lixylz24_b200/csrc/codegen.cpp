@@ -462,28 +462,32 @@ std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int
     k << "    const int k0 = warp * K;\n";
     k << "    const u32 *A = P.col[" << col_a << "], *B = P.col[" << col_b << "];\n";
     k << "    const long long lda = P.ld[" << col_a << "], ldb = P.ld[" << col_b << "];\n";
-    k << "    u64 lo[K], cor[K]; u32 hi[K]; u64 ss = 0;\n";
-    k << "#pragma unroll\n    for (int m = 0; m < K; ++m) { lo[m] = 0ull; hi[m] = 0u; cor[m] = 0ull; }\n";
+    // 96-bit carry-save column sums a0:a1:a2 (add.cc chains on the IMAD.WIDE product)
+    // split accumulators: low and high 32-bit halves of every product summed in
+    // separate u64s (2^32 additions each before overflow): no carry flags live
+    // across products, so ptxas never spills condition codes
+    k << "    u64 alo[K], ahi[K], cor[K]; u64 ss = 0;\n";
+    k << "#pragma unroll\n    for (int m = 0; m < K; ++m) { alo[m] = 0ull; ahi[m] = 0ull; cor[m] = 0ull; }\n";
     k << "    const int ilo = k0 - (LB_ - 1) > 0 ? k0 - (LB_ - 1) : 0;\n";
     k << "    const int ihi = k0 + K - 1 < LA_ - 1 ? k0 + K - 1 : LA_ - 1;\n";
+    k << "    const int ib0 = ilo - ilo % K;\n";
     k << "    const long long n = P.n;\n";
     k << "    for (long long r0 = (long long)blockIdx.x * 32; r0 < n; r0 += (long long)gridDim.x * 32) {\n";
     k << "        const long long row = r0 + lane;\n";
     k << "        if (row < n) {\n";
-    // window w[m] = B_{k0 + m - i}
-    k << "            u32 w[K];\n";
-    k << "#pragma unroll\n            for (int m = 0; m < K; ++m) { const int j = k0 + m - ilo; w[m] = (j >= 0 && j < LB_) ? __ldg(B + (long long)j * ldb + row) : 0u; }\n";
-    k << "            for (int i = ilo; i <= ihi; ++i) {\n";
-    k << "                const u32 ai = __ldg(A + (long long)i * lda + row);\n";
+    // circular window: slot (j mod K) holds B_j; at step i column m reads slot (k0+m-i) mod K
+    k << "            u32 c[K];\n";
+    k << "#pragma unroll\n            for (int m = 0; m < K; ++m) { const int j = k0 + m - ib0; c[m] = (j >= 0 && j < LB_) ? __ldg(B + (long long)j * ldb + row) : 0u; }\n";
+    k << "            for (int ib = ib0; ib <= ihi; ib += K) {\n";
+    k << "#pragma unroll\n              for (int u = 0; u < K; ++u) {\n";
+    k << "                const int i = ib + u;\n";
+    k << "                const u32 ai = (i >= ilo && i <= ihi) ? __ldg(A + (long long)i * lda + row) : 0u;\n";
     k << "#pragma unroll\n                for (int m = 0; m < K; ++m) {\n";
-    k << "                    const u64 p = (u64)ai * w[m];\n";
-    k << "                    const u64 s = lo[m] + p;\n";
-    k << "                    hi[m] += s < p ? 1u : 0u;\n";
-    k << "                    lo[m] = s;\n";
+    k << "                    u64 p; asm(\"mul.wide.u32 %0, %1, %2;\" : \"=l\"(p) : \"r\"(ai), \"r\"(c[(m - u + K) % K]));\n";
+    k << "                    alo[m] += (u32)p; ahi[m] += (u32)(p >> 32);\n";
     k << "                }\n";
-    k << "                // slide the window: w[m] <- B_{k0 + m - (i+1)}\n";
-    k << "#pragma unroll\n                for (int m = K - 1; m > 0; --m) w[m] = w[m - 1];\n";
-    k << "                { const int j = k0 - i - 1; w[0] = (j >= 0 && j < LB_) ? __ldg(B + (long long)j * ldb + row) : 0u; }\n";
+    k << "                { const int j = k0 - i - 1; c[K - 1 - u] = (j >= 0 && j < LB_) ? __ldg(B + (long long)j * ldb + row) : 0u; }\n";
+    k << "              }\n";
     k << "            }\n";
     // sign corrections
     k << "            const u32 sa = __ldg(A + (long long)(LA_ - 1) * lda + row) >> 31;\n";
@@ -493,11 +497,14 @@ std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int
     k << "            ss += sa & sb;\n";
     k << "        }\n";
     k << "    }\n";
-    // warp reduce
+    // warp reduce (value a0 + a1 2^32 + a2 2^64 per column, exact in u64 slots below)
+    // column value = alo + ahi 2^32 = lo + hi 2^64 (exact)
+    k << "    u64 lo[K], hi[K];\n";
+    k << "#pragma unroll\n    for (int m = 0; m < K; ++m) { const u64 t = alo[m] + (ahi[m] << 32); hi[m] = (ahi[m] >> 32) + (t < alo[m] ? 1ull : 0ull); lo[m] = t; }\n";
     k << "#pragma unroll\n    for (int m = 0; m < K; ++m) {\n";
     k << "#pragma unroll\n        for (int o = 16; o > 0; o >>= 1) {\n";
-    k << "            const u64 l2 = __shfl_down_sync(0xFFFFFFFFu, lo[m], o); const u32 h2 = __shfl_down_sync(0xFFFFFFFFu, hi[m], o);\n";
-    k << "            const u64 s = lo[m] + l2; hi[m] += h2 + (s < l2 ? 1u : 0u); lo[m] = s;\n";
+    k << "            const u64 l2 = __shfl_down_sync(0xFFFFFFFFu, lo[m], o); const u64 h2 = __shfl_down_sync(0xFFFFFFFFu, hi[m], o);\n";
+    k << "            const u64 s = lo[m] + l2; hi[m] += h2 + (s < l2 ? 1ull : 0ull); lo[m] = s;\n";
     k << "            cor[m] += __shfl_down_sync(0xFFFFFFFFu, cor[m], o);\n";
     k << "        }\n    }\n";
     k << "#pragma unroll\n    for (int o = 16; o > 0; o >>= 1) ss += __shfl_down_sync(0xFFFFFFFFu, ss, o);\n";
@@ -508,7 +515,7 @@ std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int
     k << "            if (col + 2 < NSL) {\n";
     k << "                if ((u32)lo[m]) atomicAdd(&pos[col], (u64)(u32)lo[m]);\n";
     k << "                if (lo[m] >> 32) atomicAdd(&pos[col + 1], lo[m] >> 32);\n";
-    k << "                if (hi[m]) atomicAdd(&pos[col + 2], (u64)hi[m]);\n";
+    k << "                if (hi[m]) atomicAdd(&pos[col + 2], hi[m]);\n";
     k << "                if ((u32)cor[m]) atomicAdd(&neg[col], (u64)(u32)cor[m]);\n";
     k << "                if (cor[m] >> 32) atomicAdd(&neg[col + 1], cor[m] >> 32);\n";
     k << "            }\n        }\n";
