@@ -312,6 +312,7 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     k += "|" + std::to_string(extra);
     if (getenv("UP_NO_OPT")) k += "|noopt";
     if (getenv("UP_NO_WIDE")) k += "|nowide";
+    if (getenv("UP_SPLIT")) k += "|split";
     return k;
 }
 
@@ -655,7 +656,9 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     if (N < cols[0].n) return fail(UP_E_INVAL, "n_global < local rows");
     // Split SUM: top-level column products -> row-contraction kernels, the
     // rest -> the fused per-thread kernel, then an exact combine (SUM is linear).
-    if (!getenv("UP_NO_SPLIT")) {
+    // opt-in (UP_SPLIT=1): measured slower than the fused per-thread kernel at
+    // p = 200 (7.5 vs 2.9 ms) and only 1.2x faster at p = 1000 in round 1
+    if (getenv("UP_SPLIT") && !getenv("UP_NO_SPLIT")) {
         Typed ts;
         if (up_status s = type_expr(expr, cols, ncols, ts)) return s;
         const int LAs = limbs_for_precision(sum_precision(ts.root->p, N));

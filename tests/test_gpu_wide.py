@@ -89,6 +89,7 @@ def test_split_sum_matches_unsplit_and_oracle(expr, types, lead, monkeypatch):
     """Row-contraction SUM (products as carry-save column sums over rows, signs
     by correction terms) + fused rest kernel + combine == oracle == UP_NO_SPLIT."""
     n = 300 if types[0][0] >= 1000 else 2000
+    monkeypatch.setenv("UP_SPLIT", "1")
     host = G.gen_cols(n, types, config=3, nonzero_lead_cols=lead, seed=11)
     want, P, S = oracle.eval_sum(expr, G.to_oracle(host, types), threads=8)
     from paper_conf_icde_lixylz24_b200 import up
@@ -97,7 +98,7 @@ def test_split_sum_matches_unsplit_and_oracle(expr, types, lead, monkeypatch):
     got = up.result_to_string(c.sum_expr(expr, cols), S)
     c.check()
     assert got == want
-    monkeypatch.setenv("UP_NO_SPLIT", "1")
+    monkeypatch.delenv("UP_SPLIT")
     c2 = up.Context(0)
     cols2 = [c2.column_from_host_bin(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
     assert up.result_to_string(c2.sum_expr(expr, cols2), S) == want
