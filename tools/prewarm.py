@@ -38,6 +38,32 @@ def sources():
         out.append(up.gen_sin_source(P, 9, 8, False, 1))
     out.append(up.gen_sin_source(2000, 9, 8, True, 40))
     out.append(up.gen_sin_source(500, 9, 8, True, 300))
+    # heavier kernels of the GPU test-suite (exact sources: LA depends on the row count)
+    for bits, n in ((1024, 333), (512, 333), (256, 333), (64, 333)):
+        N, _, _ = synth.rsa_modulus(bits)
+        for e in (3, 65537):
+            out.append(up.gen_modexp_source(e, N, len(str(N)), False, n))
+    N, _, _ = synth.rsa_modulus(1024)
+    out.append(up.gen_modexp_source(65537, N, len(str(N)), True, 10_000_000))
+    out.append(up.gen_modexp_source(65537, N, len(str(N)), False, 10_000_000))
+    for p, s in ((200, 50), (500, 75), (1000, 100)):
+        for n in (1, 9, 1000, 300, 2000, 500):
+            out.append(up.gen_source("sum", "c1*c2 - c3/c4", [(p, s)] * 4, n))
+    out.append(up.gen_source("sum", "c1*c2 - c3/c4", [(200, 50)] * 4, 12_500_000))
+    out.append(up.gen_source("sum", "c1+c2", [(35, 5), (32, 2)], 10_000_000))
+    import math
+    def q5(terms):
+        e = "c1"
+        for k in range(1, terms):
+            m = 2 * k + 1
+            e += (" - " if k % 2 else " + ") + "*".join(["c1"] * m) + "/" + str(math.factorial(m))
+        return e
+    for terms in (2, 3, 5, 8, 11):
+        out.append(up.gen_source("eval", q5(terms), [(9, 8)], 300))
+        out.append(up.gen_source("sum", q5(terms), [(9, 8)], 300))
+    for P in (1000,):
+        out.append(up.gen_sin_source(P, 9, 8, True, 1_000_000))
+        out.append(up.gen_sin_source(P, 9, 8, False, 1_000_000))
     return list(dict.fromkeys(out))
 
 
