@@ -9,9 +9,16 @@
 // 128-bit loads, intermediates in registers, SUM fused into the same kernel.
 #include "codegen.h"
 
+#include <cstdlib>
 #include <sstream>
 
 namespace uph {
+
+std::string launch_bounds(int threads) {
+    std::string s = "__launch_bounds__(" + std::to_string(threads);
+    if (const char *m = getenv("UP_MINBLOCKS")) s += std::string(", ") + std::to_string(atoi(m));
+    return s + ")";
+}
 
 namespace {
 
@@ -179,7 +186,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     const bool cs = LOUT <= 8;
     const int LA = opt.sum ? opt.LA : LOUT;
     const int NS = cs ? LOUT : LA;
-    k << "extern \"C\" __global__ void __launch_bounds__(256) upk(const up_kparams P) {\n";
+    k << "extern \"C\" __global__ void " << launch_bounds(256) << " upk(const up_kparams P) {\n";
     k << "    constexpr int R = " << R << ";\n";
     k << "    u32 fl = 0;\n";
     if (opt.sum) {

@@ -7,6 +7,10 @@
 
 namespace uph {
 
+// __launch_bounds__(threads[, UP_MINBLOCKS]) -- the env knob trades registers
+// for occupancy in experiments (part of the source, so of the cache key)
+std::string launch_bounds(int threads);
+
 struct GenOpts {
     bool sum = false;   // fused SUM (true) or per-row column output (false)
     int LA = 0;         // SUM limbs
