@@ -14,9 +14,10 @@
 
 namespace uph {
 
-std::string launch_bounds(int threads) {
+std::string launch_bounds(int threads, int min_blocks) {
     std::string s = "__launch_bounds__(" + std::to_string(threads);
-    if (const char *m = getenv("UP_MINBLOCKS")) s += std::string(", ") + std::to_string(atoi(m));
+    if (const char *m = getenv("UP_MINBLOCKS")) min_blocks = atoi(m);
+    if (min_blocks > 0) s += ", " + std::to_string(min_blocks);
     return s + ")";
 }
 
@@ -186,7 +187,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     const bool cs = LOUT <= 8;
     const int LA = opt.sum ? opt.LA : LOUT;
     const int NS = cs ? LOUT : LA;
-    k << "extern \"C\" __global__ void " << launch_bounds(256) << " upk(const up_kparams P) {\n";
+    k << "extern \"C\" __global__ void " << launch_bounds(256, R == 1 ? 2 : 0) << " upk(const up_kparams P) {\n";
     k << "    constexpr int R = " << R << ";\n";
     k << "    u32 fl = 0;\n";
     if (opt.sum) {
