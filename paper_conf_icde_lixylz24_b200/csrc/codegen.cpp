@@ -187,7 +187,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     const bool cs = LOUT <= 8;
     const int LA = opt.sum ? opt.LA : LOUT;
     const int NS = cs ? LOUT : LA;
-    k << "extern \"C\" __global__ void " << launch_bounds(256, R == 1 ? 2 : 0) << " upk(const up_kparams P) {\n";
+    k << "extern \"C\" __global__ void " << launch_bounds(256, (R == 1 && max_limbs(root) <= 64) ? 2 : 0) << " upk(const up_kparams P) {\n";
     k << "    constexpr int R = " << R << ";\n";
     k << "    u32 fl = 0;\n";
     if (opt.sum) {
