@@ -226,3 +226,86 @@ def add_strings(values: Sequence[str], p: int, s: int) -> str:
     if e:
         raise OracleError(e, "add_strings")
     return buf.value.decode()
+
+
+AGG_KINDS = ("SUM", "MIN", "MAX", "AVG")
+
+
+def _scaled_int(txt: str, s: int) -> int:
+    neg = txt.startswith("-")
+    t = txt[1:] if neg else txt
+    ip, _, fp = t.partition(".")
+    v = int(ip + fp.ljust(s, "0")[:s]) if s else int(ip)
+    return -v if neg else v
+
+
+def _fmt_scaled(v: int, s: int) -> str:
+    a = str(abs(v))
+    if s:
+        a = a.rjust(s + 1, "0")
+        a = a[:-s] + "." + a[-s:]
+    return ("-" if v < 0 else "") + a
+
+
+def agg_type(kind: str, p: int, s: int, n_global: int):
+    """Result type of an aggregate over n_global tuples, P:L1069-1080 (Sec. III-B):
+    MAX/MIN keep the expression's precision; SUM is p + ceil(log10 N) (orc_sum_type);
+    AVG follows the SUM rule and then the division rule (p1-p2+s2+5, s1+4),
+    P:L1049-1058, with the divisor converted to DECIMAL(ceil(log10 N)+1, 0)."""
+    if kind in ("MIN", "MAX"):
+        return p, s
+    ps, ss = sum_type(p, s, n_global)
+    if kind == "SUM":
+        return ps, ss
+    if kind == "AVG":
+        p2, s2 = (ps - p) + 1, 0          # ceil(log10 N) = ps - p
+        return ps - p2 + s2 + 5, ss + 4
+    raise ValueError(kind)
+
+
+def group_aggregate(aggs, cols: Sequence[Column], group=None, n_groups: int = 1, n_global: int = 0):
+    """SELECT agg(expr), ... GROUP BY g, written out row by row (Python ints on
+    the oracle's exact per-row values, orc_eval_rows).  Rows with g < 0 are
+    excluded (a WHERE filter).  AVG = trunc(SUM * 10^(s2+4) / COUNT) with s2 = 0
+    (the division of P:L1049-1058 by COUNT as DECIMAL(ceil(log10 N)+1, 0),
+    truncation toward zero, reading Q4).  An empty group reports 0 (SQL NULL,
+    see its count).  Returns ([[string per group] per aggregate], counts, types)."""
+    n = cols[0].n
+    N = n_global or n
+    gid = np.zeros(n, np.int64) if group is None else np.asarray(group, dtype=np.int64)
+    counts = [0] * n_groups
+    for g in gid.tolist():
+        if 0 <= g < n_groups:
+            counts[g] += 1
+    results, types = [], []
+    for kind, expr in aggs:
+        P, S = expr_type(expr, cols)
+        rows = eval_rows(expr, cols, strict=False)
+        acc = [None] * n_groups
+        for r, g in zip(rows, gid.tolist()):
+            if not 0 <= g < n_groups:
+                continue
+            if r.startswith("E"):
+                raise OracleError(int(r[1:] or 1), expr)
+            v = _scaled_int(r, S)
+            a = acc[g]
+            if kind in ("SUM", "AVG"):
+                acc[g] = v if a is None else a + v
+            elif kind == "MIN":
+                acc[g] = v if a is None or v < a else a
+            else:
+                acc[g] = v if a is None or v > a else a
+        tp, ts = agg_type(kind, P, S, N)
+        out = []
+        for g in range(n_groups):
+            a = acc[g]
+            if a is None:
+                out.append(_fmt_scaled(0, ts))
+            elif kind == "AVG":
+                q = abs(a) * 10 ** 4 // counts[g]
+                out.append(_fmt_scaled(-q if a < 0 else q, ts))
+            else:
+                out.append(_fmt_scaled(a, ts))
+        results.append(out)
+        types.append((tp, ts))
+    return results, counts, types
