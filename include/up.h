@@ -148,6 +148,36 @@ up_status up_sum_combine(up_ctx *ctx, const uint32_t *d_partials, int32_t nranks
                          uint32_t *d_out, void *stream);
 
 /*
+ * Grouped aggregation: SELECT agg_a(expr_a) ... GROUP BY g in
+ * ONE kernel launch.  Aggregate typing follows P:L1069-1080 (Sec. III-B):
+ *   SUM(e): DECIMAL(p + ceil(log10 N), s)      (as up_sum_type)
+ *   MIN(e), MAX(e): DECIMAL(p, s)              (the expression's type)
+ *   AVG(e): the SUM rule, then the division rule with the
+ *           divisor COUNT converted to DECIMAL(ceil(log10 N)+1, 0), i.e.
+ *           DECIMAL(p + 4, s + 4), value trunc(SUM * 10^4 / COUNT)
+ *           (truncation toward zero, reading Q4).
+ * N = n_global (0 means the local row count): the tuple count of the query.
+ * kinds[a] in up_agg_kind; exprs[a] use the up_eval_expr grammar.
+ * d_group: device int32 per row; rows with a negative id are excluded (a
+ *   WHERE filter); ids >= n_groups set the INVAL flag and are excluded; NULL
+ *   means one group (n_groups must then be 1).  n_groups is limited by the
+ *   shared-memory group records (UNSUPPORTED beyond ~200 KB per block).
+ * d_out (device, packed): aggregate a's results for groups 0..n_groups-1,
+ *   each up_agg_type(...).limbs two's-complement limbs, aggregates in order;
+ *   total sum_a n_groups * limbs_a uint32.
+ * d_counts (device): n_groups uint64 row counts (COUNT(*) per group).  An
+ *   empty group yields 0 for every aggregate (SQL NULL; see its count).
+ * Errors raised by rows of excluded groups are not flagged.  Single-GPU
+ * (MIN/MAX/AVG partials do not combine by up_sum_combine).
+ */
+typedef enum { UP_AGG_SUM = 0, UP_AGG_MIN = 1, UP_AGG_MAX = 2, UP_AGG_AVG = 3 } up_agg_kind;
+up_status up_agg_type(const char *expr, int32_t kind, const up_column *cols, int ncols, int64_t n_global,
+                      int32_t *p, int32_t *s, int32_t *limbs);
+up_status up_group_aggregate(up_ctx *ctx, int32_t n_aggs, const int32_t *kinds, const char *const *exprs,
+                             const up_column *cols, int ncols, const int32_t *d_group, int32_t n_groups,
+                             int64_t n_global, uint32_t *d_out, uint64_t *d_counts, void *stream);
+
+/*
  * x^e mod N per row (row a8; Query 4 P:L2124-2154 generalised to any e).
  * base: s == 0, values >= 0 (a negative value sets INVAL); values >= N are
  * reduced mod N first.  exponent, modulus: decimal strings, modulus odd and
@@ -208,6 +238,10 @@ up_status up_gen_contract_source(int32_t La, int32_t Lb, int32_t LA, int sign, c
 up_status up_jit_prewarm(const char *src);
 /* Generated sin_taylor source for x DECIMAL(p,s) (sum != 0: fused SUM variant). */
 up_status up_gen_sin_source(int32_t P, int32_t p, int32_t s, int sum, int64_t n_global, char *buf, size_t len);
+/* Generated grouped-aggregation source (arguments as up_group_aggregate). */
+up_status up_gen_group_agg_source(int32_t n_aggs, const int32_t *kinds, const char *const *exprs,
+                                  const up_column *cols, int ncols, int32_t n_groups, int64_t n_global,
+                                  char *buf, size_t len);
 /* Generated modexp source for a DECIMAL(base_p,0) base (sum != 0: fused SUM variant). */
 up_status up_gen_modexp_source(const char *exponent, const char *modulus, int32_t base_p, int sum,
                                int64_t n_global, char *buf, size_t len);

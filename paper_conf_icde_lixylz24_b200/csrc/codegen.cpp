@@ -251,6 +251,193 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
 
 
 // ---------------------------------------------------------------------------
+// Grouped aggregation (NEXT-4, P:L1069-1080, P:L1480-1537 moderngpu-style
+// SUM/MAX/MIN/AVG, here in ONE pass): every distinct expression is evaluated
+// once per row (shared column loads); a warp's rows of one group are combined
+// with redux.sync and merged into the block's shared-memory group record
+// (SUM: carry-save slots + negative count; MIN/MAX: best value under a lock;
+// COUNT); blocks commit SUM slots with 64-bit atomics and MIN/MAX records to
+// scratch; the last block (ticket) normalises, reduces MIN/MAX over blocks
+// and finalises AVG = trunc(SUM * 10^4 / COUNT) (the paper's division rule
+// with the divisor DECIMAL(ceil(log10 N)+1, 0): s2 = 0, so 10^(s2+4)).
+std::string gen_group_agg_kernel(const std::vector<AggItem> &aggs, const std::vector<ColType> &cols, int G,
+                                 GenInfo &info, int &mm_words) {
+    // distinct expressions
+    std::vector<const Node *> exprs;
+    std::vector<std::string> names;
+    std::vector<int> expr_of(aggs.size());
+    for (size_t a = 0; a < aggs.size(); ++a) {
+        std::string cn = canonical(aggs[a].root) + "@" + std::to_string(aggs[a].root->p) + "," + std::to_string(aggs[a].root->s);
+        size_t e = 0;
+        while (e < names.size() && names[e] != cn) ++e;
+        if (e == names.size()) { names.push_back(cn); exprs.push_back(aggs[a].root); }
+        expr_of[a] = (int)e;
+    }
+    const int NE = (int)exprs.size();
+    // slot layout per group: [0] count, then per summed expression L+1 slots
+    std::vector<int> sum_off(NE, -1);
+    int SLOTS = 1;
+    for (size_t a = 0; a < aggs.size(); ++a) {
+        const int e = expr_of[a];
+        if ((aggs[a].kind == AGG_SUM || aggs[a].kind == AGG_AVG) && sum_off[e] < 0) {
+            sum_off[e] = SLOTS;
+            SLOTS += exprs[e]->L + 1;
+        }
+    }
+    // MIN/MAX records per group: one best value per MIN/MAX aggregate
+    std::vector<int> mm_off(aggs.size(), -1), mm_idx(aggs.size(), -1);
+    int MMW = 0, NMM = 0;
+    for (size_t a = 0; a < aggs.size(); ++a)
+        if (aggs[a].kind == AGG_MIN || aggs[a].kind == AGG_MAX) {
+            mm_off[a] = MMW;
+            mm_idx[a] = NMM++;
+            MMW += exprs[expr_of[a]]->L;
+        }
+    mm_words = MMW;
+    std::vector<bool> used(cols.size(), false);
+    for (const Node *e : exprs) used_columns(e, used);
+
+    std::ostringstream k;
+    k << "// generated by libup codegen: grouped aggregation, G=" << G << "\n";
+    static const char *const kNames[] = {"SUM", "MIN", "MAX", "AVG"};
+    for (size_t a = 0; a < aggs.size(); ++a)
+        k << "//   agg " << a << ": " << kNames[aggs[a].kind] << "(" << names[(size_t)expr_of[a]] << ")\n";
+    k << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
+    for (int e = 0; e < NE; ++e) {
+        Emitter E;
+        std::string res = E.emit(exprs[e]);
+        k << "__device__ __forceinline__ void eval_" << e << "(";
+        bool first = true;
+        for (size_t c = 0; c < cols.size(); ++c) {
+            if (!used[c]) continue;
+            k << (first ? "" : ", ") << "const u32 (&x" << c << ")[" << cols[c].limbs << "]";
+            first = false;
+        }
+        k << (first ? "" : ", ") << "u32 (&res)[" << exprs[e]->L << "], u32 &fl) {\n" << E.o.str();
+        k << "    sext<" << exprs[e]->L << "," << exprs[e]->L << ">(res, " << res << ");\n}\n\n";
+    }
+    k << "constexpr int G = " << G << ", SLOTS = " << SLOTS << ", MMW = " << std::max(MMW, 1) << ", NMM = " << std::max(NMM, 1) << ";\n";
+    k << "extern \"C\" __global__ void " << launch_bounds(256) << " upk(const up_kparams P) {\n";
+    k << "    extern __shared__ __align__(16) u64 gsm[];\n";
+    k << "    u32 *gmm = reinterpret_cast<u32 *>(gsm + G * SLOTS);\n";
+    k << "    u32 *glk = gmm + G * MMW;\n";
+    k << "    for (int i = threadIdx.x; i < G * SLOTS; i += blockDim.x) gsm[i] = 0ull;\n";
+    k << "    for (int i = threadIdx.x; i < G * NMM; i += blockDim.x) glk[i] = 0u;\n";
+    if (NMM) {
+        // identity of MAX (and of MAX over complements): the most negative value
+        k << "    for (int g = threadIdx.x; g < G; g += blockDim.x) {\n";
+        for (size_t a = 0; a < aggs.size(); ++a) {
+            if (mm_off[a] < 0) continue;
+            const int L = exprs[expr_of[a]]->L;
+            k << "        for (int j = 0; j < " << L << "; ++j) gmm[g * MMW + " << mm_off[a] << " + j] = j == " << L - 1 << " ? 0x80000000u : 0u;\n";
+        }
+        k << "    }\n";
+    }
+    k << "    __syncthreads();\n";
+    k << "    const int lane = threadIdx.x & 31;\n";
+    k << "    u32 fl = 0;\n";
+    k << "    const long long n = P.n;\n";
+    k << "    const long long stride = (long long)gridDim.x * blockDim.x;\n";
+    k << "    for (long long wb = (long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31); wb < n; wb += stride) {\n";
+    k << "        const long long i = wb + lane;\n";
+    k << "        const long long ii = i < n ? i : n - 1;\n";
+    k << "        int g = i < n ? (P.group ? __ldcs(P.group + ii) : 0) : -1;\n";
+    k << "        if (g >= G) { fl |= F_INVAL; g = -1; }\n";
+    for (size_t c = 0; c < cols.size(); ++c) {
+        if (!used[c]) continue;
+        k << "        u32 x" << c << "[" << cols[c].limbs << "];\n";
+        k << "#pragma unroll\n        for (int j = 0; j < " << cols[c].limbs << "; ++j) x" << c << "[j] = __ldcs(P.col[" << c << "] + j * P.ld[" << c << "] + ii);\n";
+    }
+    k << "        u32 fr = 0;\n";
+    for (int e = 0; e < NE; ++e) {
+        k << "        u32 v" << e << "[" << exprs[e]->L << "]; eval_" << e << "(";
+        bool first = true;
+        for (size_t c = 0; c < cols.size(); ++c) {
+            if (!used[c]) continue;
+            k << (first ? "" : ", ") << "x" << c;
+            first = false;
+        }
+        k << (first ? "" : ", ") << "v" << e << ", fr);\n";
+    }
+    k << "        const bool act = g >= 0;\n";
+    k << "        if (act) fl |= fr;\n";
+    k << "        u32 pend = __ballot_sync(0xffffffffu, act);\n";
+    k << "        while (pend) {\n";
+    k << "            const int ldr = __ffs(pend) - 1;\n";
+    k << "            const int gl = __shfl_sync(0xffffffffu, g, ldr);\n";
+    k << "            const bool mine = act && g == gl;\n";
+    k << "            const u32 peers = __ballot_sync(0xffffffffu, mine);\n";
+    k << "            pend &= ~peers;\n";
+    k << "            if (mine) {\n";
+    k << "                u64 *gs = gsm + gl * SLOTS;\n";
+    k << "                const bool lead = lane == ldr;\n";
+    k << "                if (lead) atomicAdd(&gs[0], (u64)__popc(peers));\n";
+    for (int e = 0; e < NE; ++e)
+        if (sum_off[e] >= 0) k << "                grp_sum_update<" << exprs[e]->L << ">(v" << e << ", peers, lead, gs + " << sum_off[e] << ");\n";
+    for (size_t a = 0; a < aggs.size(); ++a) {
+        if (mm_off[a] < 0) continue;
+        const int e = expr_of[a], L = exprs[e]->L;
+        k << "                { u32 w[" << L << "];\n#pragma unroll\n                  for (int j = 0; j < " << L << "; ++j) w[j] = "
+          << (aggs[a].kind == AGG_MAX ? "" : "~") << "v" << e << "[j];\n";
+        k << "                  grp_max_update<" << L << ">(w, peers, lane, gmm + gl * MMW + " << mm_off[a] << ", glk + gl * NMM + " << mm_idx[a] << "); }\n";
+    }
+    k << "            }\n        }\n    }\n";
+    k << "    if (fl) atomicOr(P.flags, fl);\n";
+    k << "    __syncthreads();\n";
+    k << "    for (int i = threadIdx.x; i < G * SLOTS; i += blockDim.x) { const u64 t = gsm[i]; if (t) atomicAdd(&P.ws[i], t); }\n";
+    if (NMM) k << "    for (int i = threadIdx.x; i < G * MMW; i += blockDim.x) P.scratch[(long long)blockIdx.x * G * MMW + i] = gmm[i];\n";
+    k << "    __threadfence();\n    __syncthreads();\n";
+    k << "    __shared__ u32 s_last;\n";
+    k << "    if (threadIdx.x == 0) s_last = (atomicAdd(P.ticket, 1u) == gridDim.x - 1) ? 1u : 0u;\n";
+    k << "    __syncthreads();\n    if (!s_last) return;\n    __threadfence();\n";
+    k << "    for (int i = threadIdx.x; i < G * SLOTS; i += blockDim.x) gsm[i] = atomicExch(&P.ws[i], 0ull);\n";
+    k << "    __syncthreads();\n";
+    k << "    if (threadIdx.x == 0) *P.ticket = 0u;\n";
+    k << "    for (int g = threadIdx.x; g < G; g += blockDim.x) P.counts[g] = gsm[g * SLOTS];\n";
+    k << "    for (int t = threadIdx.x; t < " << aggs.size() << " * G; t += blockDim.x) {\n";
+    k << "        const int a = t / G, g = t - a * G;\n";
+    k << "        const u64 *gs = gsm + g * SLOTS;\n";
+    k << "        const u64 cnt = gs[0];\n";
+    k << "        switch (a) {\n";
+    for (size_t a = 0; a < aggs.size(); ++a) {
+        const int e = expr_of[a], L = exprs[e]->L, LA = aggs[a].LA, Lr = aggs[a].Lr;
+        k << "        case " << a << ": {\n";
+        k << "            u32 *o = P.result + " << aggs[a].off << "ll + (long long)g * " << Lr << ";\n";
+        if (aggs[a].kind == AGG_SUM) {
+            k << "            u32 r[" << LA << "]; slots_to_limbs<" << L << "," << LA << ">(r, gs + " << sum_off[e] << ");\n";
+            k << "            for (int j = 0; j < " << Lr << "; ++j) o[j] = r[j];\n";
+        } else if (aggs[a].kind == AGG_AVG) {
+            // Q = sign * trunc(|SUM| * 10^4 / COUNT)  (P:L1076-1080 with the P:L1049-1058 quotient)
+            k << "            u32 sm_[" << LA << "]; slots_to_limbs<" << L << "," << LA << ">(sm_, gs + " << sum_off[e] << ");\n";
+            k << "            u32 ng; u32 ab[" << LA << "]; abs_copy(ab, sm_, ng);\n";
+            k << "            u32 u[" << LA + 1 << "]; mul_1<" << LA << ">(u, ab, 10000u);\n";
+            k << "            const u32 dv[2] = {(u32)cnt, (u32)(cnt >> 32)};\n";
+            k << "            u32 q[" << Lr << "], rr[2];\n";
+            k << "            if (cnt) { divmod_mag<" << LA + 1 << ",2," << Lr << ",false>(q, rr, u, dv); cond_neg(q, ng); } else zero(q);\n";
+            k << "            for (int j = 0; j < " << Lr << "; ++j) o[j] = q[j];\n";
+        } else {
+            k << "            u32 b[" << L << "];\n";
+            k << "            for (int j = 0; j < " << L << "; ++j) b[j] = j == " << L - 1 << " ? 0x80000000u : 0u;\n";
+            k << "            for (unsigned blk = 0; blk < gridDim.x; ++blk) {\n";
+            k << "                const u32 *c = P.scratch + (long long)blk * G * MMW + g * MMW + " << mm_off[a] << ";\n";
+            k << "                u32 w[" << L << "];\n";
+            k << "                for (int j = 0; j < " << L << "; ++j) w[j] = c[j];\n";
+            k << "                if (gt_signed<" << L << ">(w, b)) for (int j = 0; j < " << L << "; ++j) b[j] = w[j];\n";
+            k << "            }\n";
+            k << "            for (int j = 0; j < " << L << "; ++j) o[j] = cnt ? " << (aggs[a].kind == AGG_MAX ? "b[j]" : "~b[j]") << " : 0u;\n";
+        }
+        k << "            break; }\n";
+    }
+    k << "        }\n    }\n}\n";
+    info.rows_per_thread = 1;
+    info.threads = 256;
+    info.ws_slots = G * SLOTS;
+    info.dyn_smem = (int)(((size_t)G * SLOTS * 8 + (size_t)G * std::max(MMW, 1) * 4 + (size_t)G * std::max(NMM, 1) * 4 + 15) & ~(size_t)15);
+    return k.str();
+}
+
+
+// ---------------------------------------------------------------------------
 // Wide SUM regime (rows a10/a11 at ~40+ limbs, cfg3 DECIMAL(500..1000,...)):
 // SELECT SUM(sum_t +-term_t) = sum_t +-10^(s_out - s_t) SUM(term_t) exactly
 // (alignment is an exact x10^k and SUM is linear), so each term is summed on

@@ -35,6 +35,19 @@ bool split_sum_terms(const Node *root, const std::vector<ColType> &cols, int min
 // wide SUM regime (warp per row); "" if the expression does not fit it
 std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &cols, int LA, GenInfo &info);
 
+// grouped aggregation (NEXT-4): SUM / MIN / MAX / AVG of expressions per group
+enum AggKind { AGG_SUM = 0, AGG_MIN = 1, AGG_MAX = 2, AGG_AVG = 3 };
+struct AggItem {
+    int kind;
+    const Node *root;   // typed (optimised) expression
+    int LA;             // SUM limbs (SUM / AVG)
+    int Lr;             // result limbs
+    long long off;      // u32 offset of this aggregate's [G][Lr] block in the packed output
+};
+// mm_words: u32 words of one block's MIN/MAX record (x G x grid = scratch)
+std::string gen_group_agg_kernel(const std::vector<AggItem> &aggs, const std::vector<ColType> &cols, int G,
+                                 GenInfo &info, int &mm_words);
+
 // modexp / sin_taylor specialisations (special.cpp)
 struct ModexpPlan {
     int n = 0;          // modulus limbs

@@ -768,6 +768,145 @@ up_status up_format_decimal(const uint32_t *limbs, int32_t nlimbs, int32_t s, ch
     return UP_OK;
 }
 
+// ---- grouped aggregation (NEXT-4): typing P:L1069-1080
+}  // extern "C"
+namespace {
+
+struct AggPlan {
+    std::vector<Typed> typed;
+    std::vector<std::unique_ptr<Node>> opt;
+    std::vector<AggItem> items;
+    std::vector<ColType> types;
+    long long words = 0;   // packed output words
+    int mm_words = 0;      // MIN/MAX words per group record
+    std::string key;
+};
+
+// result type of one aggregate over N tuples
+up_status agg_result_type(int kind, const Node *root, long long N, int &p, int &s, int &LA) {
+    const int ps = sum_precision(root->p, N);   // SUM: p + ceil(log10 N)
+    LA = 0;
+    switch (kind) {
+    case AGG_SUM: p = ps; s = root->s; LA = limbs_for_precision(ps); return UP_OK;
+    case AGG_MIN: case AGG_MAX: p = root->p; s = root->s; return UP_OK;
+    case AGG_AVG: {
+        // SUM rule, then the division rule with the divisor DECIMAL(ceil(log10 N)+1, 0):
+        // (p1 - p2 + s2 + 5, s1 + 4)
+        const int pd = (ps - root->p) + 1, sd = 0;
+        p = ps - pd + sd + 5;
+        s = root->s + 4;
+        LA = limbs_for_precision(ps);
+        return UP_OK;
+    }
+    default: return fail(UP_E_INVAL, "unknown aggregate kind %d", kind);
+    }
+}
+
+up_status agg_plan(int32_t n_aggs, const int32_t *kinds, const char *const *exprs, const up_column *cols, int ncols,
+                   long long N, int G, AggPlan &pl) {
+    if (n_aggs < 1 || n_aggs > 32 || !kinds || !exprs) return fail(UP_E_INVAL, "need 1..32 aggregates");
+    if (G < 1) return fail(UP_E_INVAL, "n_groups must be >= 1");
+    pl.typed.resize((size_t)n_aggs);
+    pl.key = "gagg|" + std::to_string(G) + "|" + std::to_string(N);
+    for (int i = 0; i < ncols; ++i) pl.key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
+    if (getenv("UP_NO_OPT")) pl.key += "|noopt";
+    for (int a = 0; a < n_aggs; ++a) {
+        Typed &t = pl.typed[(size_t)a];
+        if (up_status st = type_expr(exprs[a], cols, ncols, t)) return st;
+        if (a == 0) pl.types = t.types;
+        int p = 0, s = 0, LA = 0;
+        if (up_status st = agg_result_type(kinds[a], t.root.get(), N, p, s, LA)) return st;
+        std::unique_ptr<Node> o = getenv("UP_NO_OPT") ? nullptr : optimize(t.root.get(), t.types);
+        const Node *r = o ? o.get() : t.root.get();
+        pl.opt.push_back(std::move(o));
+        AggItem it;
+        it.kind = kinds[a];
+        it.root = r;
+        it.LA = LA;
+        it.Lr = limbs_for_precision(p);
+        it.off = pl.words;
+        pl.words += (long long)G * it.Lr;
+        if (it.kind == AGG_MIN || it.kind == AGG_MAX) pl.mm_words += r->L;
+        pl.items.push_back(it);
+        pl.key += "|" + std::to_string(kinds[a]) + ":" + exprs[a];
+    }
+    return UP_OK;
+}
+
+}  // namespace
+extern "C" {
+
+up_status up_agg_type(const char *expr, int32_t kind, const up_column *cols, int ncols, int64_t n_global, int32_t *p,
+                      int32_t *s, int32_t *limbs) {
+    Typed t;
+    if (up_status st = type_expr(expr, cols, ncols, t)) return st;
+    const long long N = n_global > 0 ? n_global : (ncols ? cols[0].n : 0);
+    int pp = 0, ss = 0, LA = 0;
+    if (up_status st = agg_result_type(kind, t.root.get(), N, pp, ss, LA)) return st;
+    if (p) *p = pp;
+    if (s) *s = ss;
+    if (limbs) *limbs = limbs_for_precision(pp);
+    return UP_OK;
+}
+
+up_status up_group_aggregate(up_ctx *c, int32_t n_aggs, const int32_t *kinds, const char *const *exprs,
+                             const up_column *cols, int ncols, const int32_t *d_group, int32_t n_groups,
+                             int64_t n_global, uint32_t *d_out, uint64_t *d_counts, void *stream) {
+    if (!c || !cols || ncols < 1 || !d_out || !d_counts) return fail(UP_E_INVAL, "need a ctx, columns, d_out and d_counts");
+    for (int i = 0; i < ncols; ++i) {
+        if (up_status s = check_column(&cols[i], "input")) return s;
+        if (cols[i].n != cols[0].n) return fail(UP_E_INVAL, "columns differ in length");
+    }
+    if (!d_group && n_groups != 1) return fail(UP_E_INVAL, "d_group == NULL needs n_groups == 1");
+    const long long N = n_global > 0 ? n_global : cols[0].n;
+    if (N < cols[0].n) return fail(UP_E_INVAL, "n_global < local rows");
+    AggPlan pl;
+    if (up_status s = agg_plan(n_aggs, kinds, exprs, cols, ncols, N, n_groups, pl)) return s;
+    std::lock_guard<std::mutex> g(c->mu);
+    JitKernel *k = nullptr;
+    int mmw = 0;
+    if (up_status s = kernel_for(c, pl.key, [&](GenInfo &info) {
+            std::string src = gen_group_agg_kernel(pl.items, pl.types, n_groups, info, mmw);
+            if (info.dyn_smem > 200 * 1024) { fail(UP_E_UNSUPPORTED, "too many groups for one block's records"); return std::string(); }
+            return src; }, &k))
+        return s;
+    up_kparams P;
+    fill_cols(P, cols, ncols);
+    P.ws = c->d_ws;
+    P.ticket = c->d_ticket;
+    P.flags = c->d_flags;
+    P.result = d_out;
+    P.group = d_group;
+    P.counts = (unsigned long long *)d_counts;
+    if (pl.mm_words) {
+        const long long want = (P.n + k->threads - 1) / k->threads;
+        const long long grid = std::max(1ll, std::min(want, (long long)k->blocks_per_sm * c->num_sms));
+        void *sp = nullptr;
+        const size_t bytes = (size_t)grid * (size_t)n_groups * (size_t)pl.mm_words * 4;
+        if (bytes > c->scratch_bytes) {
+            if (c->d_scratch) { CUDA_TRY(cudaDeviceSynchronize()); CUDA_TRY(cudaFree(c->d_scratch)); c->d_scratch = nullptr; }
+            CUDA_TRY(cudaMalloc(&c->d_scratch, bytes));
+            c->scratch_bytes = bytes;
+        }
+        sp = c->d_scratch;
+        P.scratch = (unsigned int *)sp;
+    }
+    return launch(c, k, P, std::max(P.n, 1ll), (cudaStream_t)stream);
+}
+
+up_status up_gen_group_agg_source(int32_t n_aggs, const int32_t *kinds, const char *const *exprs, const up_column *cols,
+                                  int ncols, int32_t n_groups, int64_t n_global, char *buf, size_t len) {
+    AggPlan pl;
+    const long long N = n_global > 0 ? n_global : (ncols ? cols[0].n : 0);
+    if (up_status s = agg_plan(n_aggs, kinds, exprs, cols, ncols, N, n_groups, pl)) return s;
+    GenInfo info;
+    int mmw = 0;
+    std::string src = gen_group_agg_kernel(pl.items, pl.types, n_groups, info, mmw);
+    if (!buf || src.size() + 1 > len) return fail(UP_E_NOMEM, "need %zu bytes", src.size() + 1);
+    memcpy(buf, src.c_str(), src.size() + 1);
+    return UP_OK;
+}
+
 // ---- diagnostics (no GPU needed): generated source and an NVRTC-only compile
 up_status up_gen_source(const char *variant, const char *expr, const up_column *cols, int ncols, int64_t n_global,
                         char *buf, size_t len) {

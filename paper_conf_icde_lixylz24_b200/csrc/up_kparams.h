@@ -16,4 +16,6 @@ typedef struct {
     unsigned int *flags;                   /* sticky error flags (F_*) */
     unsigned int *scratch;                 /* per-thread global scratch (sin_P running sums) */
     long long scratch_stride;              /* elements between consecutive words of one thread */
+    const int *group;                      /* group_aggregate: group id per row (NULL = one group) */
+    unsigned long long *counts;            /* group_aggregate: rows per group */
 } up_kparams;

@@ -39,7 +39,10 @@ EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_l
            "up_sin_taylor", "up_sin_taylor_sum", "up_check", "up_format_decimal", "up_launch_count",
            "up_jit_ms", "up_gen_source", "up_nvrtc_compile", "up_gen_modexp_source", "up_jit_prewarm", "up_gen_sin_source", "up_compact_bytes",
            "up_column_from_host_compact", "up_column_from_device_compact", "up_column_to_host_compact",
-           "up_expr_optimized", "up_gen_contract_source"]
+           "up_expr_optimized", "up_gen_contract_source", "up_agg_type", "up_group_aggregate",
+           "up_gen_group_agg_source"]
+
+AGG = {"SUM": 0, "MIN": 1, "MAX": 2, "AVG": 3}
 
 
 def lib():
@@ -89,6 +92,12 @@ def lib():
     L.up_column_from_device_compact.argtypes = [P, P, PC, P]
     L.up_column_to_host_compact.argtypes = [P, PC, P, P]
     L.up_gen_sin_source.argtypes = [c.c_int32, c.c_int32, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
+    PI32 = c.POINTER(c.c_int32)
+    L.up_agg_type.argtypes = [c.c_char_p, c.c_int32, PC, c.c_int, c.c_int64, PI32, PI32, PI32]
+    L.up_group_aggregate.argtypes = [P, c.c_int32, PI32, c.POINTER(c.c_char_p), PC, c.c_int, P, c.c_int32,
+                                     c.c_int64, P, P, P]
+    L.up_gen_group_agg_source.argtypes = [c.c_int32, PI32, c.POINTER(c.c_char_p), PC, c.c_int, c.c_int32,
+                                          c.c_int64, c.c_char_p, c.c_size_t]
     L.up_gen_modexp_source.argtypes = [c.c_char_p, c.c_char_p, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
     _lib = L
     return L
@@ -375,8 +384,62 @@ class Context:
         _chk(lib().up_sin_taylor_sum(self.h, ctypes.byref(xd), P, n_global, out.data_ptr(), _stream_ptr(stream)))
         return out
 
+    def group_aggregate(self, aggs: Sequence[tuple], cols: Sequence[Column], group=None, n_groups: int = 1,
+                        n_global: int = 0, out=None, counts=None, stream=None):
+        """SELECT agg(expr), ... GROUP BY group in one launch (include/up.h
+        up_group_aggregate).  aggs: [(kind, expr)], kind in AGG's keys.
+        Returns (packed int32 device tensor, int64 device counts, layout) where
+        layout[a] = (p, s, limbs, offset) and aggregate a of group g occupies
+        out[offset + g*limbs : offset + (g+1)*limbs]."""
+        import torch
+        layout, off = [], 0
+        for kind, expr in aggs:
+            p, s, L = agg_type(kind, expr, [c.type() for c in cols], n_global or cols[0].n)
+            layout.append((p, s, L, off))
+            off += n_groups * L
+        dev = cols[0].data.device
+        if out is None:
+            out = torch.empty(max(off, 1), dtype=torch.int32, device=dev)
+        if counts is None:
+            counts = torch.empty(n_groups, dtype=torch.int64, device=dev)
+        kinds, exprs = _agg_args(aggs)
+        _chk(lib().up_group_aggregate(self.h, len(aggs), kinds, exprs, _descs(cols), len(cols),
+                                      group.data_ptr() if group is not None else None, n_groups, n_global,
+                                      out.data_ptr(), counts.data_ptr(), _stream_ptr(stream)))
+        return out, counts, layout
+
     def check(self, stream=None):
         _chk(lib().up_check(self.h, _stream_ptr(stream)))
+
+
+def _agg_args(aggs):
+    kinds = (ctypes.c_int32 * len(aggs))(*[AGG[k] for k, _ in aggs])
+    exprs = (ctypes.c_char_p * len(aggs))(*[e.encode() for _, e in aggs])
+    return kinds, exprs
+
+
+def _type_descs(types: Sequence[tuple], n: int = 1):
+    arr = (up_column * max(1, len(types)))()
+    for i, (p, s) in enumerate(types):
+        arr[i] = up_column(n, ld_for(n), p, s, limbs(p), 0, None)
+    return arr
+
+
+def agg_type(kind: str, expr: str, types: Sequence[tuple], n_global: int):
+    """(p, s, limbs) of an aggregate over n_global tuples (no GPU)."""
+    p, s, L = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    _chk(lib().up_agg_type(expr.encode(), AGG[kind], _type_descs(types), len(types), n_global,
+                           ctypes.byref(p), ctypes.byref(s), ctypes.byref(L)))
+    return p.value, s.value, L.value
+
+
+def group_results(out, counts, layout, n_groups: int):
+    """Packed group_aggregate output -> ([[string per group] per aggregate], [count per group])."""
+    host = out.detach().cpu().tolist()
+    res = []
+    for p, s, L, off in layout:
+        res.append([format_decimal(host[off + g * L: off + (g + 1) * L], s) for g in range(n_groups)])
+    return res, [int(x) for x in counts.detach().cpu().tolist()]
 
 
 def _fmt(v: int, s: int) -> str:
@@ -430,6 +493,14 @@ def expr_optimized(expr: str, types: Sequence[tuple]) -> str:
 def gen_contract_source(La: int, Lb: int, LA: int, sign: int = 1) -> str:
     buf = ctypes.create_string_buffer(1 << 20)
     _chk(lib().up_gen_contract_source(La, Lb, LA, sign, buf, len(buf)))
+    return buf.value.decode()
+
+
+def gen_group_agg_source(aggs: Sequence[tuple], types: Sequence[tuple], n_groups: int, n_global: int) -> str:
+    kinds, exprs = _agg_args(aggs)
+    buf = ctypes.create_string_buffer(1 << 24)
+    _chk(lib().up_gen_group_agg_source(len(aggs), kinds, exprs, _type_descs(types, n_global), len(types),
+                                       n_groups, n_global, buf, len(buf)))
     return buf.value.decode()
 
 

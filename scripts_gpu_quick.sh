@@ -11,4 +11,10 @@ fi
 for c in $BENCH; do
   timeout 900 python bench.py $BENCH_ARGS --config $c > gpurun_out/bench_q_cfg$c.log 2>&1; echo "bench rc=$?" >> gpurun_out/bench_q_cfg$c.log
 done
+if [ -n "$Q1" ]; then
+  timeout 900 python tools/bench_q1.py > gpurun_out/q1.log 2>&1; echo "q1 rc=$?" >> gpurun_out/q1.log
+fi
+if [ -n "$OPS" ]; then
+  timeout 900 python tools/bench_operators.py > gpurun_out/ops.log 2>&1; echo "ops rc=$?" >> gpurun_out/ops.log
+fi
 echo done

@@ -95,3 +95,20 @@ def test_specialised_kernels_compile_for_sm100a(variant, expr, types, tmp_path):
     assert (tmp_path / "k.cubin").stat().st_size > 0
     if expr == "c1+c2":
         assert spills == 0 and regs <= 64, log
+
+
+def test_group_aggregate_typing_and_kernel_compile(tmp_path):
+    """NEXT-4: aggregate typing on the host and the generated
+    grouped-aggregation kernel compiles for sm_100a without spills."""
+    t = [(12, 2), (12, 2), (3, 2), (3, 2)]
+    N = 60_000_000
+    assert up.agg_type("SUM", "c1", t, N)[:2] == (12 + 8, 2)
+    assert up.agg_type("MIN", "c2*(1-c3)", t, N)[:2] == up.agg_type("MAX", "c2*(1-c3)", t, N)[:2]
+    p, s, _ = up.agg_type("SUM", "c2*(1-c3)", t, N)
+    assert up.agg_type("MAX", "c2*(1-c3)", t, N)[:2] == (p - 8, s)
+    assert up.agg_type("AVG", "c3", t, N)[:2] == (3 + 4, 2 + 4)
+    aggs = [("SUM", "c1"), ("AVG", "c2*(1-c3)*(1+c4)"), ("MIN", "c1-c2"), ("MAX", "c3")]
+    src = up.gen_group_agg_source(aggs, t, 4, N)
+    log = up.nvrtc_compile(src, str(tmp_path / "g.cubin"))
+    regs, spills = _regs(log)
+    assert spills == 0, log

@@ -64,6 +64,12 @@ def sources():
     for P in (1000,):
         out.append(up.gen_sin_source(P, 9, 8, True, 1_000_000))
         out.append(up.gen_sin_source(P, 9, 8, False, 1_000_000))
+    # TPC-H Q1-shaped grouped aggregation (tools/bench_q1.py, 60M rows)
+    q1 = [("SUM", "c1"), ("SUM", "c2"), ("SUM", "c2*(1-c3)"), ("SUM", "c2*(1-c3)*(1+c4)"),
+          ("AVG", "c1"), ("AVG", "c2"), ("AVG", "c3")]
+    out.append(up.gen_group_agg_source(q1, [(12, 2)] * 4, 4, 60_000_000))
+    for P in (18, 38, 76, 153, 307):
+        out.append(up.gen_group_agg_source(q1, [(P, 2), (P, 2), (3, 2), (3, 2)], 4, 60_000_000))
     return list(dict.fromkeys(out))
 
 
