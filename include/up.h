@@ -158,7 +158,7 @@ up_status up_sum_combine(up_ctx *ctx, const uint32_t *d_partials, int32_t nranks
  *           (truncation toward zero, reading Q4).
  * N = n_global (0 means the local row count): the tuple count of the query.
  * kinds[a] in up_agg_kind; exprs[a] use the up_eval_expr grammar.
- * d_group: device int32 per row; rows with a negative id are excluded (a
+ * d_group: device int32 per row (16-byte aligned); rows with a negative id are excluded (a
  *   WHERE filter); ids >= n_groups set the INVAL flag and are excluded; NULL
  *   means one group (n_groups must then be 1).  n_groups is limited by the
  *   shared-memory group records (UNSUPPORTED beyond ~200 KB per block).

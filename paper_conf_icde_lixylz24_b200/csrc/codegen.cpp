@@ -251,15 +251,23 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
 
 
 // ---------------------------------------------------------------------------
-// Grouped aggregation (NEXT-4, P:L1069-1080, P:L1480-1537 moderngpu-style
-// SUM/MAX/MIN/AVG, here in ONE pass): every distinct expression is evaluated
-// once per row (shared column loads); a warp's rows of one group are combined
-// with redux.sync and merged into the block's shared-memory group record
-// (SUM: carry-save slots + negative count; MIN/MAX: best value under a lock;
-// COUNT); blocks commit SUM slots with 64-bit atomics and MIN/MAX records to
-// scratch; the last block (ticket) normalises, reduces MIN/MAX over blocks
-// and finalises AVG = trunc(SUM * 10^4 / COUNT) (the paper's division rule
-// with the divisor DECIMAL(ceil(log10 N)+1, 0): s2 = 0, so 10^(s2+4)).
+// Grouped aggregation (NEXT-4; the paper's moderngpu multi-pass
+// SUM/MAX/MIN/AVG of P:L1480-1537 becomes ONE pass): every distinct
+// expression is evaluated once per row (shared column loads) and folded into
+// its group's record:
+//   private mode (records fit shared memory per thread): each thread owns a
+//     record per group in shared memory ([slot][thread] layout, conflict-free)
+//     -- one 64-bit add per limb per row, no atomics, no warp collectives;
+//     4 rows per thread with 128-bit loads when every operand is narrow;
+//   warp mode (wide records): a warp's rows of one group are combined with
+//     redux.sync and merged into a per-block record (smem atomics; MIN/MAX
+//     under a per-record lock).
+// Record: SUM = carry-save slots + negative count; MIN/MAX = best value (MIN
+// as MAX of the bitwise complement); COUNT.  Blocks commit SUM slots with
+// 64-bit atomics and MIN/MAX records to scratch; the last block (ticket)
+// normalises, reduces MIN/MAX over blocks and finalises
+// AVG = trunc(SUM * 10^4 / COUNT) (division rule with the divisor
+// DECIMAL(ceil(log10 N)+1, 0): s2 = 0, so 10^(s2+4)).
 std::string gen_group_agg_kernel(const std::vector<AggItem> &aggs, const std::vector<ColType> &cols, int G,
                                  GenInfo &info, int &mm_words) {
     // distinct expressions
@@ -296,9 +304,32 @@ std::string gen_group_agg_kernel(const std::vector<AggItem> &aggs, const std::ve
     mm_words = MMW;
     std::vector<bool> used(cols.size(), false);
     for (const Node *e : exprs) used_columns(e, used);
+    int maxL = 0;
+    bool divmod = false;
+    for (const Node *e : exprs) { maxL = std::max(maxL, max_limbs(e)); divmod = divmod || uses_divmod(e); }
+
+    // private records: T threads x G x (SLOTS u64 + MMW u32) within ~110 KB (2 blocks / SM)
+    const size_t per_thread = (size_t)G * ((size_t)SLOTS * 8 + (size_t)MMW * 4);
+    // block size maximising resident threads per SM under the 228 KB of shared
+    // memory (1 KB reserved per block); measured on B200: more resident warps
+    // beat larger blocks (Q1 shape: T = 32 0.80 ms vs T = 128 0.89 ms)
+    int T = 0, best_threads = 0;
+    for (int t : {256, 128, 64, 32}) {
+        const size_t blk = per_thread * (size_t)t + 1024;
+        const int nb = std::min<int>({32, 2048 / t, (int)((228u * 1024u) / blk)});
+        if (nb >= 1 && per_thread * (size_t)t <= 220 * 1024 && nb * t >= best_threads) { best_threads = nb * t; T = t; }
+    }
+    if (const char *e = getenv("UP_GAGG_T")) {   // experiment: force T private records (<= 220 KB)
+        const int t = atoi(e);
+        T = (t == 32 || t == 64 || t == 128 || t == 256) && per_thread * (size_t)t <= 220 * 1024 ? t : 0;
+    }
+    if (getenv("UP_GAGG_WARP")) T = 0;
+    const bool priv = T > 0;
+    const int R = priv && maxL <= 8 && !divmod ? 4 : 1;
+    if (!priv) T = 256;
 
     std::ostringstream k;
-    k << "// generated by libup codegen: grouped aggregation, G=" << G << "\n";
+    k << "// generated by libup codegen: grouped aggregation, G=" << G << (priv ? " (private records)" : " (warp records)") << "\n";
     static const char *const kNames[] = {"SUM", "MIN", "MAX", "AVG"};
     for (size_t a = 0; a < aggs.size(); ++a)
         k << "//   agg " << a << ": " << kNames[aggs[a].kind] << "(" << names[(size_t)expr_of[a]] << ")\n";
@@ -316,85 +347,184 @@ std::string gen_group_agg_kernel(const std::vector<AggItem> &aggs, const std::ve
         k << (first ? "" : ", ") << "u32 (&res)[" << exprs[e]->L << "], u32 &fl) {\n" << E.o.str();
         k << "    sext<" << exprs[e]->L << "," << exprs[e]->L << ">(res, " << res << ");\n}\n\n";
     }
-    k << "constexpr int G = " << G << ", SLOTS = " << SLOTS << ", MMW = " << std::max(MMW, 1) << ", NMM = " << std::max(NMM, 1) << ";\n";
-    k << "extern \"C\" __global__ void " << launch_bounds(256) << " upk(const up_kparams P) {\n";
-    k << "    extern __shared__ __align__(16) u64 gsm[];\n";
-    k << "    u32 *gmm = reinterpret_cast<u32 *>(gsm + G * SLOTS);\n";
-    k << "    u32 *glk = gmm + G * MMW;\n";
-    k << "    for (int i = threadIdx.x; i < G * SLOTS; i += blockDim.x) gsm[i] = 0ull;\n";
-    k << "    for (int i = threadIdx.x; i < G * NMM; i += blockDim.x) glk[i] = 0u;\n";
-    if (NMM) {
-        // identity of MAX (and of MAX over complements): the most negative value
-        k << "    for (int g = threadIdx.x; g < G; g += blockDim.x) {\n";
-        for (size_t a = 0; a < aggs.size(); ++a) {
-            if (mm_off[a] < 0) continue;
-            const int L = exprs[expr_of[a]]->L;
-            k << "        for (int j = 0; j < " << L << "; ++j) gmm[g * MMW + " << mm_off[a] << " + j] = j == " << L - 1 << " ? 0x80000000u : 0u;\n";
-        }
-        k << "    }\n";
-    }
-    k << "    __syncthreads();\n";
-    k << "    const int lane = threadIdx.x & 31;\n";
-    k << "    u32 fl = 0;\n";
-    k << "    const long long n = P.n;\n";
-    k << "    const long long stride = (long long)gridDim.x * blockDim.x;\n";
-    k << "    for (long long wb = (long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31); wb < n; wb += stride) {\n";
-    k << "        const long long i = wb + lane;\n";
-    k << "        const long long ii = i < n ? i : n - 1;\n";
-    k << "        int g = i < n ? (P.group ? __ldcs(P.group + ii) : 0) : -1;\n";
-    k << "        if (g >= G) { fl |= F_INVAL; g = -1; }\n";
-    for (size_t c = 0; c < cols.size(); ++c) {
-        if (!used[c]) continue;
-        k << "        u32 x" << c << "[" << cols[c].limbs << "];\n";
-        k << "#pragma unroll\n        for (int j = 0; j < " << cols[c].limbs << "; ++j) x" << c << "[j] = __ldcs(P.col[" << c << "] + j * P.ld[" << c << "] + ii);\n";
-    }
-    k << "        u32 fr = 0;\n";
-    for (int e = 0; e < NE; ++e) {
-        k << "        u32 v" << e << "[" << exprs[e]->L << "]; eval_" << e << "(";
+    auto eval_one = [&](int e, const char *ind, const char *row) {
+        k << ind << "u32 v" << e << "[" << exprs[e]->L << "]; eval_" << e << "(";
         bool first = true;
         for (size_t c = 0; c < cols.size(); ++c) {
             if (!used[c]) continue;
-            k << (first ? "" : ", ") << "x" << c;
+            k << (first ? "" : ", ") << "x" << c << row;
             first = false;
         }
         k << (first ? "" : ", ") << "v" << e << ", fr);\n";
+    };
+    k << "constexpr int G = " << G << ", SLOTS = " << SLOTS << ", MMW = " << std::max(MMW, 1) << ", NMM = " << std::max(NMM, 1)
+      << ", T = " << T << ", R = " << R << ";\n";
+    k << "extern \"C\" __global__ void " << launch_bounds(T) << " upk(const up_kparams P) {\n";
+    k << "    extern __shared__ __align__(16) u64 gsm[];\n";
+    k << "    const int tid = threadIdx.x;\n";
+    k << "    u32 fl = 0;\n";
+    k << "    const long long n = P.n;\n";
+    if (priv) {
+        // ---------------- private mode: [slot][thread] records
+        k << "    u32 *gmm = reinterpret_cast<u32 *>(gsm + (long long)G * SLOTS * T);\n";
+        k << "    for (int q = 0; q < G * SLOTS; ++q) gsm[q * T + tid] = 0ull;\n";
+        if (NMM) {
+            k << "    for (int g = 0; g < G; ++g) {\n";
+            for (size_t a = 0; a < aggs.size(); ++a) {
+                if (mm_off[a] < 0) continue;
+                const int L = exprs[expr_of[a]]->L;
+                k << "        for (int j = 0; j < " << L << "; ++j) gmm[(g * MMW + " << mm_off[a] << " + j) * T + tid] = j == " << L - 1 << " ? 0x80000000u : 0u;\n";
+            }
+            k << "    }\n";
+        }
+        k << "    const long long stride = (long long)gridDim.x * T * R;\n";
+        k << "    for (long long base = ((long long)blockIdx.x * T + tid) * R; base < n; base += stride) {\n";
+        k << "        int gi[R];\n";
+        if (R == 4) {
+            k << "        if (!P.group) { gi[0] = gi[1] = gi[2] = gi[3] = 0; }\n";
+            k << "        else if (base + 3 < n) { const int4 q = __ldcs(reinterpret_cast<const int4 *>(P.group + base)); gi[0] = q.x; gi[1] = q.y; gi[2] = q.z; gi[3] = q.w; }\n";
+            k << "        else { for (int r = 0; r < 4; ++r) gi[r] = base + r < n ? P.group[base + r] : -1; }\n";
+        } else {
+            k << "        gi[0] = P.group ? __ldcs(P.group + base) : 0;\n";
+        }
+        for (size_t c = 0; c < cols.size(); ++c) {
+            if (!used[c]) continue;
+            const int Lc = cols[c].limbs;
+            k << "        u32 x" << c << "[R][" << Lc << "];\n";
+            k << "        { const u32 *p = P.col[" << c << "] + base; const long long ld = P.ld[" << c << "];\n";
+            if (R == 4)
+                k << "#pragma unroll\n          for (int j = 0; j < " << Lc << "; ++j) { const uint4 v = __ldcs(reinterpret_cast<const uint4 *>(p + j * ld));"
+                     " x" << c << "[0][j] = v.x; x" << c << "[1][j] = v.y; x" << c << "[2][j] = v.z; x" << c << "[3][j] = v.w; } }\n";
+            else
+                k << "#pragma unroll\n          for (int j = 0; j < " << Lc << "; ++j) x" << c << "[0][j] = __ldcs(p + j * ld); }\n";
+        }
+        k << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n";
+        k << "            int g = base + r < n ? gi[r] : -1;\n";
+        k << "            if (g >= G) { fl |= F_INVAL; g = -1; }\n";
+        k << "            u32 fr = 0;\n";
+        k << "            u64 *rec = gsm + (long long)(g < 0 ? 0 : g) * SLOTS * T + tid;\n";
+        k << "            if (g >= 0) rec[0] += 1ull;\n";
+        for (int e = 0; e < NE; ++e) {
+            eval_one(e, "            ", "[r]");
+            k << "            if (g >= 0) {\n";
+            if (sum_off[e] >= 0) {
+                const int L = exprs[e]->L;
+                k << "#pragma unroll\n                for (int j = 0; j < " << L << "; ++j) rec[(" << sum_off[e] << " + j) * T] += v" << e << "[j];\n";
+                k << "                rec[" << sum_off[e] + L << " * T] += v" << e << "[" << L - 1 << "] >> 31;\n";
+            }
+            for (size_t a = 0; a < aggs.size(); ++a) {
+                if (mm_off[a] < 0 || expr_of[a] != e) continue;
+                const int L = exprs[e]->L;
+                const char *inv = aggs[a].kind == AGG_MAX ? "" : "~";
+                k << "                { u32 *b = gmm + (g * MMW + " << mm_off[a] << ") * T + tid; u32 w[" << L << "], cur[" << L << "];\n";
+                k << "#pragma unroll\n                  for (int j = 0; j < " << L << "; ++j) { w[j] = " << inv << "v" << e << "[j]; cur[j] = b[j * T]; }\n";
+                k << "                  if (gt_signed<" << L << ">(w, cur)) {\n#pragma unroll\n                    for (int j = 0; j < " << L << "; ++j) b[j * T] = w[j]; } }\n";
+            }
+            k << "            }\n";
+        }
+        k << "            if (g >= 0) fl |= fr;\n";
+        k << "        }\n    }\n";
+        k << "    if (fl) atomicOr(P.flags, fl);\n";
+        k << "    __syncthreads();\n";
+        // block totals: slot q summed over the T records (rotated start: conflict-free)
+        k << "    for (int q = tid; q < G * SLOTS; q += T) {\n";
+        k << "        u64 t = 0;\n";
+        k << "        for (int i = 0; i < T; ++i) t += gsm[q * T + ((i + tid) & (T - 1))];\n";
+        k << "        if (t) atomicAdd(&P.ws[q], t);\n    }\n";
+        if (NMM) {
+            k << "    for (int q = tid; q < G * NMM; q += T) {\n";
+            k << "        const int g = q / NMM, m = q - g * NMM;\n";
+            k << "        switch (m) {\n";
+            for (size_t a = 0; a < aggs.size(); ++a) {
+                if (mm_off[a] < 0) continue;
+                const int L = exprs[expr_of[a]]->L;
+                k << "        case " << mm_idx[a] << ": {\n";
+                k << "            const u32 *b = gmm + (g * MMW + " << mm_off[a] << ") * T;\n";
+                k << "            u32 best[" << L << "], w[" << L << "];\n";
+                k << "            for (int j = 0; j < " << L << "; ++j) best[j] = b[j * T];\n";
+                k << "            for (int i = 1; i < T; ++i) {\n";
+                k << "                for (int j = 0; j < " << L << "; ++j) w[j] = b[j * T + i];\n";
+                k << "                if (gt_signed<" << L << ">(w, best)) for (int j = 0; j < " << L << "; ++j) best[j] = w[j];\n";
+                k << "            }\n";
+                k << "            u32 *o = P.scratch + (long long)blockIdx.x * G * MMW + g * MMW + " << mm_off[a] << ";\n";
+                k << "            for (int j = 0; j < " << L << "; ++j) o[j] = best[j];\n";
+                k << "            break; }\n";
+            }
+            k << "        }\n    }\n";
+        }
+        k << "    __syncthreads();\n";
+    } else {
+        // ---------------- warp mode: per-block records, warp-combined updates
+        k << "    u32 *gmm = reinterpret_cast<u32 *>(gsm + G * SLOTS);\n";
+        k << "    u32 *glk = gmm + G * MMW;\n";
+        k << "    for (int i = tid; i < G * SLOTS; i += blockDim.x) gsm[i] = 0ull;\n";
+        k << "    for (int i = tid; i < G * NMM; i += blockDim.x) glk[i] = 0u;\n";
+        if (NMM) {
+            k << "    for (int g = tid; g < G; g += blockDim.x) {\n";
+            for (size_t a = 0; a < aggs.size(); ++a) {
+                if (mm_off[a] < 0) continue;
+                const int L = exprs[expr_of[a]]->L;
+                k << "        for (int j = 0; j < " << L << "; ++j) gmm[g * MMW + " << mm_off[a] << " + j] = j == " << L - 1 << " ? 0x80000000u : 0u;\n";
+            }
+            k << "    }\n";
+        }
+        k << "    __syncthreads();\n";
+        k << "    const int lane = tid & 31;\n";
+        k << "    const long long stride = (long long)gridDim.x * blockDim.x;\n";
+        k << "    for (long long wb = (long long)blockIdx.x * blockDim.x + (tid & ~31); wb < n; wb += stride) {\n";
+        k << "        const long long i = wb + lane;\n";
+        k << "        const long long ii = i < n ? i : n - 1;\n";
+        k << "        int g = i < n ? (P.group ? __ldcs(P.group + ii) : 0) : -1;\n";
+        k << "        if (g >= G) { fl |= F_INVAL; g = -1; }\n";
+        for (size_t c = 0; c < cols.size(); ++c) {
+            if (!used[c]) continue;
+            k << "        u32 x" << c << "[" << cols[c].limbs << "];\n";
+            k << "#pragma unroll\n        for (int j = 0; j < " << cols[c].limbs << "; ++j) x" << c << "[j] = __ldcs(P.col[" << c << "] + j * P.ld[" << c << "] + ii);\n";
+        }
+        k << "        u32 fr = 0;\n";
+        k << "        const bool act = g >= 0;\n";
+        // pass -1: COUNT; pass e: expression e (evaluated just before its pass: one value live at a time)
+        for (int e = -1; e < NE; ++e) {
+            if (e >= 0) eval_one(e, "        ", "");
+            k << "        for (u32 pend = __ballot_sync(0xffffffffu, act); pend; ) {\n";
+            k << "            const int ldr = __ffs(pend) - 1;\n";
+            k << "            const int gl = __shfl_sync(0xffffffffu, g, ldr);\n";
+            k << "            const bool mine = act && g == gl;\n";
+            k << "            const u32 peers = __ballot_sync(0xffffffffu, mine);\n";
+            k << "            pend &= ~peers;\n";
+            k << "            if (mine) {\n";
+            k << "                u64 *gs = gsm + gl * SLOTS;\n";
+            k << "                const bool lead = lane == ldr;\n";
+            if (e < 0) k << "                if (lead) atomicAdd(&gs[0], (u64)__popc(peers));\n";
+            else {
+                if (sum_off[e] >= 0) k << "                grp_sum_update<" << exprs[e]->L << ">(v" << e << ", peers, lead, gs + " << sum_off[e] << ");\n";
+                for (size_t a = 0; a < aggs.size(); ++a) {
+                    if (mm_off[a] < 0 || expr_of[a] != e) continue;
+                    const int L = exprs[e]->L;
+                    k << "                { u32 w[" << L << "];\n#pragma unroll\n                  for (int j = 0; j < " << L << "; ++j) w[j] = "
+                      << (aggs[a].kind == AGG_MAX ? "" : "~") << "v" << e << "[j];\n";
+                    k << "                  grp_max_update<" << L << ">(w, peers, lane, gmm + gl * MMW + " << mm_off[a] << ", glk + gl * NMM + " << mm_idx[a] << "); }\n";
+                }
+            }
+            k << "            }\n        }\n";
+        }
+        k << "        if (act) fl |= fr;\n";
+        k << "    }\n";
+        k << "    if (fl) atomicOr(P.flags, fl);\n";
+        k << "    __syncthreads();\n";
+        k << "    for (int i = tid; i < G * SLOTS; i += blockDim.x) { const u64 t = gsm[i]; if (t) atomicAdd(&P.ws[i], t); }\n";
+        if (NMM) k << "    for (int i = tid; i < G * MMW; i += blockDim.x) P.scratch[(long long)blockIdx.x * G * MMW + i] = gmm[i];\n";
     }
-    k << "        const bool act = g >= 0;\n";
-    k << "        if (act) fl |= fr;\n";
-    k << "        u32 pend = __ballot_sync(0xffffffffu, act);\n";
-    k << "        while (pend) {\n";
-    k << "            const int ldr = __ffs(pend) - 1;\n";
-    k << "            const int gl = __shfl_sync(0xffffffffu, g, ldr);\n";
-    k << "            const bool mine = act && g == gl;\n";
-    k << "            const u32 peers = __ballot_sync(0xffffffffu, mine);\n";
-    k << "            pend &= ~peers;\n";
-    k << "            if (mine) {\n";
-    k << "                u64 *gs = gsm + gl * SLOTS;\n";
-    k << "                const bool lead = lane == ldr;\n";
-    k << "                if (lead) atomicAdd(&gs[0], (u64)__popc(peers));\n";
-    for (int e = 0; e < NE; ++e)
-        if (sum_off[e] >= 0) k << "                grp_sum_update<" << exprs[e]->L << ">(v" << e << ", peers, lead, gs + " << sum_off[e] << ");\n";
-    for (size_t a = 0; a < aggs.size(); ++a) {
-        if (mm_off[a] < 0) continue;
-        const int e = expr_of[a], L = exprs[e]->L;
-        k << "                { u32 w[" << L << "];\n#pragma unroll\n                  for (int j = 0; j < " << L << "; ++j) w[j] = "
-          << (aggs[a].kind == AGG_MAX ? "" : "~") << "v" << e << "[j];\n";
-        k << "                  grp_max_update<" << L << ">(w, peers, lane, gmm + gl * MMW + " << mm_off[a] << ", glk + gl * NMM + " << mm_idx[a] << "); }\n";
-    }
-    k << "            }\n        }\n    }\n";
-    k << "    if (fl) atomicOr(P.flags, fl);\n";
-    k << "    __syncthreads();\n";
-    k << "    for (int i = threadIdx.x; i < G * SLOTS; i += blockDim.x) { const u64 t = gsm[i]; if (t) atomicAdd(&P.ws[i], t); }\n";
-    if (NMM) k << "    for (int i = threadIdx.x; i < G * MMW; i += blockDim.x) P.scratch[(long long)blockIdx.x * G * MMW + i] = gmm[i];\n";
+    // ---------------- common tail: last block normalises and finalises
     k << "    __threadfence();\n    __syncthreads();\n";
     k << "    __shared__ u32 s_last;\n";
-    k << "    if (threadIdx.x == 0) s_last = (atomicAdd(P.ticket, 1u) == gridDim.x - 1) ? 1u : 0u;\n";
+    k << "    if (tid == 0) s_last = (atomicAdd(P.ticket, 1u) == gridDim.x - 1) ? 1u : 0u;\n";
     k << "    __syncthreads();\n    if (!s_last) return;\n    __threadfence();\n";
-    k << "    for (int i = threadIdx.x; i < G * SLOTS; i += blockDim.x) gsm[i] = atomicExch(&P.ws[i], 0ull);\n";
+    k << "    for (int i = tid; i < G * SLOTS; i += blockDim.x) gsm[i] = atomicExch(&P.ws[i], 0ull);\n";
     k << "    __syncthreads();\n";
-    k << "    if (threadIdx.x == 0) *P.ticket = 0u;\n";
-    k << "    for (int g = threadIdx.x; g < G; g += blockDim.x) P.counts[g] = gsm[g * SLOTS];\n";
-    k << "    for (int t = threadIdx.x; t < " << aggs.size() << " * G; t += blockDim.x) {\n";
+    k << "    if (tid == 0) *P.ticket = 0u;\n";
+    k << "    for (int g = tid; g < G; g += blockDim.x) P.counts[g] = gsm[g * SLOTS];\n";
+    k << "    for (int t = tid; t < " << aggs.size() << " * G; t += blockDim.x) {\n";
     k << "        const int a = t / G, g = t - a * G;\n";
     k << "        const u64 *gs = gsm + g * SLOTS;\n";
     k << "        const u64 cnt = gs[0];\n";
@@ -429,10 +559,15 @@ std::string gen_group_agg_kernel(const std::vector<AggItem> &aggs, const std::ve
         k << "            break; }\n";
     }
     k << "        }\n    }\n}\n";
-    info.rows_per_thread = 1;
-    info.threads = 256;
+    info.rows_per_thread = R;
+    info.threads = T;
     info.ws_slots = G * SLOTS;
-    info.dyn_smem = (int)(((size_t)G * SLOTS * 8 + (size_t)G * std::max(MMW, 1) * 4 + (size_t)G * std::max(NMM, 1) * 4 + 15) & ~(size_t)15);
+    if (priv)
+        info.dyn_smem = (int)((per_thread * (size_t)T + 15) & ~(size_t)15);
+    else
+        info.dyn_smem = (int)(((size_t)G * SLOTS * 8 + (size_t)G * std::max(MMW, 1) * 4 + (size_t)G * std::max(NMM, 1) * 4 + 15) & ~(size_t)15);
+    // the last block re-reads G * SLOTS slots into gsm: the smem must hold them
+    info.dyn_smem = std::max(info.dyn_smem, (int)(((size_t)G * SLOTS * 8 + 15) & ~(size_t)15));
     return k.str();
 }
 

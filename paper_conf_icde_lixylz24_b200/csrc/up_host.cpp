@@ -364,7 +364,7 @@ up_status expr_kernel(up_ctx *c, const char *expr, const up_column *cols, int nc
     k->rows_per_block = info.rows_per_block;
     if (info.threads != k->threads || info.dyn_smem != k->dyn_smem) {
         k->threads = info.threads;
-        if (info.dyn_smem > 48 * 1024)
+        if (info.dyn_smem > 0)
             CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, info.dyn_smem));
         k->dyn_smem = info.dyn_smem;
         int nb = 0;
@@ -392,7 +392,7 @@ up_status kernel_for(up_ctx *c, const std::string &key, Gen gen, JitKernel **out
     k->rows_per_block = info.rows_per_block;
     if (info.threads != k->threads || info.dyn_smem != k->dyn_smem) {
         k->threads = info.threads;
-        if (info.dyn_smem > 48 * 1024)
+        if (info.dyn_smem > 0)
             CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, info.dyn_smem));
         k->dyn_smem = info.dyn_smem;
         int nb = 0;
@@ -810,6 +810,8 @@ up_status agg_plan(int32_t n_aggs, const int32_t *kinds, const char *const *expr
     pl.key = "gagg|" + std::to_string(G) + "|" + std::to_string(N);
     for (int i = 0; i < ncols; ++i) pl.key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
     if (getenv("UP_NO_OPT")) pl.key += "|noopt";
+    if (getenv("UP_GAGG_WARP")) pl.key += "|warp";
+    if (const char *e = getenv("UP_GAGG_T")) pl.key += std::string("|T") + e;
     for (int a = 0; a < n_aggs; ++a) {
         Typed &t = pl.typed[(size_t)a];
         if (up_status st = type_expr(exprs[a], cols, ncols, t)) return st;
@@ -858,6 +860,7 @@ up_status up_group_aggregate(up_ctx *c, int32_t n_aggs, const int32_t *kinds, co
         if (cols[i].n != cols[0].n) return fail(UP_E_INVAL, "columns differ in length");
     }
     if (!d_group && n_groups != 1) return fail(UP_E_INVAL, "d_group == NULL needs n_groups == 1");
+    if ((uintptr_t)d_group & 15) return fail(UP_E_INVAL, "d_group must be 16-byte aligned device memory");
     const long long N = n_global > 0 ? n_global : cols[0].n;
     if (N < cols[0].n) return fail(UP_E_INVAL, "n_global < local rows");
     AggPlan pl;
@@ -1001,7 +1004,7 @@ up_status up_internal_compile(up_ctx *c, const std::string &src, int rows_per_th
     k->ws_slots = ws_slots;
     if (threads != k->threads || dyn_smem != k->dyn_smem) {
         k->threads = threads;
-        if (dyn_smem > 48 * 1024)
+        if (dyn_smem > 0)
             CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, dyn_smem));
         k->dyn_smem = dyn_smem;
         int nb = 0;

@@ -394,7 +394,7 @@ class Context:
         import torch
         layout, off = [], 0
         for kind, expr in aggs:
-            p, s, L = agg_type(kind, expr, [c.type() for c in cols], n_global or cols[0].n)
+            p, s, L = agg_type(kind, expr, [(c.p, c.s) for c in cols], n_global or cols[0].n)
             layout.append((p, s, L, off))
             off += n_groups * L
         dev = cols[0].data.device
