@@ -14,6 +14,12 @@
 
 namespace uph {
 
+// experiment knob: UP_MUL28=1 switches expression multiplies to radix-2^28
+// product scanning (up_dev.cuh mul_mag28).  Measured on B200: cfg3 p = 200
+// 4.41e9 vs 4.66e9 rows/s for the 32-bit operand scanning (kept default),
+// p = 500 +2%.  modexp uses radix 2^28 unconditionally (special.cpp).
+std::string mul_variant_define() { return getenv("UP_MUL28") ? "#define UP_MUL28 1\n" : ""; }
+
 std::string launch_bounds(int threads, int min_blocks) {
     std::string s = "__launch_bounds__(" + std::to_string(threads);
     if (const char *m = getenv("UP_MINBLOCKS")) min_blocks = atoi(m);
@@ -171,7 +177,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
 
     std::ostringstream k;
     k << "// generated by libup codegen: " << canonical(root) << "  type (" << root->p << "," << root->s << ") L=" << LOUT << "\n";
-    k << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
+    k << mul_variant_define() << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
     // per-row evaluation with everything in registers
     k << "__device__ __forceinline__ void eval_row(";
     bool first = true;
@@ -333,7 +339,7 @@ std::string gen_group_agg_kernel(const std::vector<AggItem> &aggs, const std::ve
     static const char *const kNames[] = {"SUM", "MIN", "MAX", "AVG"};
     for (size_t a = 0; a < aggs.size(); ++a)
         k << "//   agg " << a << ": " << kNames[aggs[a].kind] << "(" << names[(size_t)expr_of[a]] << ")\n";
-    k << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
+    k << mul_variant_define() << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
     for (int e = 0; e < NE; ++e) {
         Emitter E;
         std::string res = E.emit(exprs[e]);
@@ -616,7 +622,7 @@ std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &co
     std::ostringstream k;
     k << "// generated by libup codegen (wide SUM regime): " << canonical(root) << "  type (" << root->p << "," << root->s
       << ") LA=" << LA << "\n";
-    k << "#include \"up_dev.cuh\"\n#include \"up_wide.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
+    k << mul_variant_define() << "#include \"up_dev.cuh\"\n#include \"up_wide.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
     // smem plan (in u32 words; u64 slot arrays first for alignment)
     int slot_words = 0;
     std::vector<int> slot_off(terms.size()), slot_n(terms.size());
@@ -785,7 +791,7 @@ std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int
     std::ostringstream k;
     k << "// generated by libup: row contraction SUM(c" << col_a + 1 << "*c" << col_b + 1 << ") La=" << La << " Lb=" << Lb
       << " K=" << K << " ranges=" << CR << "\n";
-    k << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
+    k << mul_variant_define() << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
     k << "extern \"C\" __global__ void __launch_bounds__(" << CR * 32 << ") upk(const up_kparams P) {\n";
     k << "    constexpr int LA_ = " << La << ", LB_ = " << Lb << ", K = " << K << ", NSL = " << NSL << ";\n";
     k << "    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n";

@@ -10,6 +10,7 @@ namespace uph {
 // __launch_bounds__(threads[, UP_MINBLOCKS]) -- the env knob trades registers
 // for occupancy in experiments (part of the source, so of the cache key)
 std::string launch_bounds(int threads, int min_blocks = 0);
+std::string mul_variant_define();
 
 struct GenOpts {
     bool sum = false;   // fused SUM (true) or per-row column output (false)

@@ -313,6 +313,7 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     if (getenv("UP_NO_OPT")) k += "|noopt";
     if (getenv("UP_NO_WIDE")) k += "|nowide";
     if (getenv("UP_SPLIT")) k += "|split";
+    if (getenv("UP_MUL28")) k += "|mul28";
     if (const char *m = getenv("UP_MINBLOCKS")) k += std::string("|mb") + m;
     return k;
 }
