@@ -178,6 +178,42 @@ up_status up_group_aggregate(up_ctx *ctx, int32_t n_aggs, const int32_t *kinds, 
                              int64_t n_global, uint32_t *d_out, uint64_t *d_counts, void *stream);
 
 /*
+ * WHERE lhs <op> rhs (the DECIMAL comparison
+ * operators of P:L730-734 Sec. II-C).  lhs, rhs: expressions over cols (the
+ * up_eval_expr grammar); op: "<" "<=" ">" ">=" "=" ("==") "<>" ("!=").  The
+ * comparison is exact: the sign of lhs - rhs evaluated at the type the
+ * paper's +/- rule gives the difference (each side keeps its
+ * own division truncation, reading Q4).  d_ids: device int32 per row; every
+ * row whose predicate is FALSE gets -1, other entries are left unchanged, so
+ * successive calls AND their predicates and the array feeds up_group_ids /
+ * up_group_aggregate (negative id = excluded).  One fused kernel launch.
+ * Rows that raise DIVZERO/OVERFLOW flag it; their predicate is unspecified.
+ */
+up_status up_filter(up_ctx *ctx, const char *lhs, const char *op, const char *rhs, const up_column *cols,
+                    int ncols, int32_t *d_ids, void *stream);
+
+/*
+ * GROUP BY key columns (DECIMAL values
+ * are compared to sort for grouping).  keys: nkeys DECIMAL columns of n rows
+ * each, compared lexicographically (keys[0] most significant), each by its
+ * exact value (one column = one scale, so by its mantissa).  d_ids: device
+ * int32 per row, IN/OUT: rows with a negative entry on input are excluded
+ * (e.g. by up_filter; pass an array of zeros to keep all rows) and stay -1;
+ * every other row receives its dense group id, 0 for the smallest key and
+ * increasing with the key.  *n_groups (host) = number of groups; the call
+ * synchronises the stream to read it.  d_first (device int64, optional,
+ * n entries): d_first[g] = the smallest row index of group g, for
+ * g < *n_groups.  Implementation: stable LSD radix sort (CUB
+ * DeviceRadixSort, one pass per 32-bit limb, least significant key column
+ * and limb first, the top limb's sign bit flipped so two's complement orders
+ * as signed; excluded rows sorted last), an adjacent-difference pass over all
+ * limbs, a prefix sum and a scatter.  Scratch: ~20 bytes per row
+ * (stream-ordered allocations).
+ */
+up_status up_group_ids(up_ctx *ctx, const up_column *keys, int nkeys, int32_t *d_ids, int64_t *n_groups,
+                       int64_t *d_first, void *stream);
+
+/*
  * x^e mod N per row (row a8; Query 4 P:L2124-2154 generalised to any e).
  * base: s == 0, values >= 0 (a negative value sets INVAL); values >= N are
  * reduced mod N first.  exponent, modulus: decimal strings, modulus odd and

@@ -309,3 +309,65 @@ def group_aggregate(aggs, cols: Sequence[Column], group=None, n_groups: int = 1,
         results.append(out)
         types.append((tp, ts))
     return results, counts, types
+
+
+CMP_OPS = ("<", "<=", ">", ">=", "=", "==", "<>", "!=")
+
+
+def _cmp(a, b, op: str) -> bool:
+    return {"<": a < b, "<=": a <= b, ">": a > b, ">=": a >= b, "=": a == b, "==": a == b,
+            "<>": a != b, "!=": a != b}[op]
+
+
+def filter_ids(lhs: str, op: str, rhs: str, cols: Sequence[Column], ids=None):
+    """WHERE lhs <op> rhs (the DECIMAL comparison operators of
+    P:L730-734).  Each side is evaluated exactly by the oracle (orc_eval_rows,
+    the paper's typing and truncation) and the two VALUES are compared as
+    exact rationals (each side's mantissa over 10^scale), written out row by
+    row.  Returns ids with -1 for every row whose predicate is false (rows
+    already negative stay negative).  Rows with an evaluation error raise."""
+    from fractions import Fraction
+    n = cols[0].n
+    out = [0] * n if ids is None else [int(v) for v in ids]
+    _, sl = expr_type(lhs, cols)
+    _, sr = expr_type(rhs, cols)
+    a_rows = eval_rows(lhs, cols, strict=False)
+    b_rows = eval_rows(rhs, cols, strict=False)
+    for i, (a, b) in enumerate(zip(a_rows, b_rows)):
+        if a.startswith("E") or b.startswith("E"):
+            raise OracleError(1, f"row {i}: evaluation error")
+        va = Fraction(_scaled_int(a, sl), 10 ** sl)
+        vb = Fraction(_scaled_int(b, sr), 10 ** sr)
+        if not _cmp(va, vb, op):
+            out[i] = -1
+    return out
+
+
+def group_ids(keys: Sequence[Column], ids=None):
+    """GROUP BY keys (DECIMAL values compared to
+    sort for grouping), written out plainly: every included row's key tuple
+    (exact values, first key most significant) is collected, the distinct
+    tuples are sorted ascending (Python's sort: a library primitive), and each
+    row gets the index of its tuple.  Rows with a negative id on input are
+    excluded and keep -1.  Returns (ids, n_groups, first) with first[g] the
+    smallest row index of group g."""
+    from fractions import Fraction
+    n = keys[0].n
+    base = [0] * n if ids is None else [int(v) for v in ids]
+    vals = []
+    for col in keys:
+        rows = eval_rows("c1", [col], strict=True)
+        vals.append([Fraction(_scaled_int(r, col.s), 10 ** col.s) for r in rows])
+    tuples = [tuple(v[i] for v in vals) for i in range(n)]
+    distinct = sorted({tuples[i] for i in range(n) if base[i] >= 0})
+    index = {t: g for g, t in enumerate(distinct)}
+    out = [-1] * n
+    first = [None] * len(distinct)
+    for i in range(n):
+        if base[i] < 0:
+            continue
+        g = index[tuples[i]]
+        out[i] = g
+        if first[g] is None:
+            first[g] = i
+    return out, len(distinct), first

@@ -215,7 +215,8 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
             k << "#pragma unroll\n          for (int j = 0; j < " << Lc << "; ++j) x" << c << "[0][j] = __ldcs(p + j * ld); }\n";
         }
     }
-    if (!opt.sum) k << "        u32 res[R][" << LOUT << "];\n";
+    const bool store = !opt.sum && !opt.cmp;
+    if (store) k << "        u32 res[R][" << LOUT << "];\n";
     k << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n";
     k << "            u32 fr = 0; u32 v[" << LOUT << "];\n";
     k << "            eval_row(";
@@ -226,10 +227,17 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
         first = false;
     }
     k << (first ? "" : ", ") << "v, fr);\n";
-    k << "            if (base + r < n) { fl |= fr;" << (opt.sum ? " acc.add(v);" : "") << " }\n";
-    if (!opt.sum) k << "#pragma unroll\n            for (int j = 0; j < " << LOUT << "; ++j) res[r][j] = v[j];\n";
+    if (opt.cmp) {
+        // WHERE: exact sign of lhs - rhs (P:L730-734 comparison operators)
+        static const char *pred[] = {"", "ng", "ng || z", "!ng && !z", "!ng", "z", "!z"};
+        k << "            if (base + r < n) { fl |= fr; const bool ng = (v[" << LOUT - 1 << "] >> 31) != 0u; const bool z = is_zero(v);\n";
+        k << "              if (!(" << pred[opt.cmp] << ")) reinterpret_cast<int *>(P.out)[base + r] = -1; }\n";
+    } else {
+        k << "            if (base + r < n) { fl |= fr;" << (opt.sum ? " acc.add(v);" : "") << " }\n";
+    }
+    if (store) k << "#pragma unroll\n            for (int j = 0; j < " << LOUT << "; ++j) res[r][j] = v[j];\n";
     k << "        }\n";
-    if (!opt.sum) {
+    if (store) {
         if (R == 4)
             k << "#pragma unroll\n        for (int j = 0; j < " << LOUT << "; ++j) __stcs(reinterpret_cast<uint4 *>(P.out + j * P.ld_out + base), make_uint4(res[0][j], res[1][j], res[2][j], res[3][j]));\n";
         else

@@ -15,7 +15,10 @@ std::string mul_variant_define();
 struct GenOpts {
     bool sum = false;   // fused SUM (true) or per-row column output (false)
     int LA = 0;         // SUM limbs
+    int cmp = 0;        // > 0: WHERE predicate sign(root) <op> 0 (CmpOp), rows that fail get id -1 in P.out
 };
+// comparison operators of up_filter (the root is lhs - rhs)
+enum CmpOp { CMP_LT = 1, CMP_LE, CMP_GT, CMP_GE, CMP_EQ, CMP_NE };
 
 struct GenInfo {
     int rows_per_thread = 1;

@@ -643,6 +643,46 @@ up_status up_eval_expr(up_ctx *c, const char *expr, const up_column *cols, int n
     return launch(c, k, P, P.n, (cudaStream_t)stream);
 }
 
+up_status up_filter(up_ctx *c, const char *lhs, const char *op, const char *rhs, const up_column *cols, int ncols,
+                    int32_t *d_ids, void *stream) {
+    if (!c || !cols || ncols < 1 || (!d_ids && cols[0].n > 0) || !lhs || !rhs || !op)
+        return fail(UP_E_INVAL, "need a ctx, columns, both sides, an operator and d_ids");
+    for (int i = 0; i < ncols; ++i) {
+        if (up_status s = check_column(&cols[i], "input")) return s;
+        if (cols[i].n != cols[0].n) return fail(UP_E_INVAL, "columns differ in length");
+    }
+    const std::string o(op);
+    int cmp = 0;
+    if (o == "<") cmp = CMP_LT;
+    else if (o == "<=") cmp = CMP_LE;
+    else if (o == ">") cmp = CMP_GT;
+    else if (o == ">=") cmp = CMP_GE;
+    else if (o == "=" || o == "==") cmp = CMP_EQ;
+    else if (o == "<>" || o == "!=") cmp = CMP_NE;
+    else return fail(UP_E_INVAL, "unknown comparison operator '%s'", op);
+    // the exact difference lhs - rhs, typed by the paper's rules:
+    // its sign decides every comparison
+    const std::string diff = "(" + std::string(lhs) + ") - (" + std::string(rhs) + ")";
+    std::lock_guard<std::mutex> g(c->mu);
+    Typed t;
+    if (up_status s = type_expr(diff.c_str(), cols, ncols, t)) return s;
+    JitKernel *k = nullptr;
+    const std::string key = key_of("cmp", diff.c_str(), cols, ncols, cmp);
+    auto gen = [&](GenInfo &info) {
+        std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(t.root.get(), t.types);
+        GenOpts go;
+        go.cmp = cmp;
+        return gen_expr_kernel(opt_root ? opt_root.get() : t.root.get(), t.types, go, info);
+    };
+    if (up_status s = kernel_for(c, key, gen, &k)) return s;
+    up_kparams P;
+    fill_cols(P, cols, ncols);
+    P.out = reinterpret_cast<uint32_t *>(d_ids);
+    P.flags = c->d_flags;
+    if (P.n == 0) return UP_OK;
+    return launch(c, k, P, P.n, (cudaStream_t)stream);
+}
+
 up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int ncols, int64_t n_global,
                       uint32_t *d_partial, void *stream) {
     if (!c || !cols || ncols < 1 || !d_partial) return fail(UP_E_INVAL, "need a ctx, columns and d_partial");
@@ -1038,3 +1078,7 @@ up_status up_internal_scratch(up_ctx *c, size_t bytes, void **out) {
     return UP_OK;
 }
 up_status up_internal_fail(up_status st, const std::string &msg) { return fail(st, "%s", msg.c_str()); }
+
+void up_internal_add_launches(up_ctx *c, long long k) {
+    if (c) c->launches += (uint64_t)k;
+}

@@ -40,7 +40,7 @@ EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_l
            "up_jit_ms", "up_gen_source", "up_nvrtc_compile", "up_gen_modexp_source", "up_jit_prewarm", "up_gen_sin_source", "up_compact_bytes",
            "up_column_from_host_compact", "up_column_from_device_compact", "up_column_to_host_compact",
            "up_expr_optimized", "up_gen_contract_source", "up_agg_type", "up_group_aggregate",
-           "up_gen_group_agg_source"]
+           "up_gen_group_agg_source", "up_filter", "up_group_ids"]
 
 AGG = {"SUM": 0, "MIN": 1, "MAX": 2, "AVG": 3}
 
@@ -98,6 +98,8 @@ def lib():
                                      c.c_int64, P, P, P]
     L.up_gen_group_agg_source.argtypes = [c.c_int32, PI32, c.POINTER(c.c_char_p), PC, c.c_int, c.c_int32,
                                           c.c_int64, c.c_char_p, c.c_size_t]
+    L.up_filter.argtypes = [P, c.c_char_p, c.c_char_p, c.c_char_p, PC, c.c_int, P, P]
+    L.up_group_ids.argtypes = [P, PC, c.c_int, P, c.POINTER(c.c_int64), P, P]
     L.up_gen_modexp_source.argtypes = [c.c_char_p, c.c_char_p, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
     _lib = L
     return L
@@ -407,6 +409,31 @@ class Context:
                                       group.data_ptr() if group is not None else None, n_groups, n_global,
                                       out.data_ptr(), counts.data_ptr(), _stream_ptr(stream)))
         return out, counts, layout
+
+    def filter(self, lhs: str, op: str, rhs: str, cols: Sequence[Column], ids=None, stream=None):
+        """WHERE lhs <op> rhs (include/up.h up_filter): rows whose predicate is
+        false get id -1 in `ids` (int32 device tensor, created as zeros when
+        None); returns ids.  Successive calls AND their predicates."""
+        import torch
+        if ids is None:
+            ids = torch.zeros(cols[0].n, dtype=torch.int32, device=cols[0].data.device)
+        _chk(lib().up_filter(self.h, lhs.encode(), op.encode(), rhs.encode(), _descs(cols), len(cols),
+                             ids.data_ptr(), _stream_ptr(stream)))
+        return ids
+
+    def group_ids(self, keys: Sequence[Column], ids=None, first: bool = False, stream=None):
+        """GROUP BY keys (include/up.h up_group_ids): dense group ids in ascending
+        key order written into `ids` (rows already negative stay excluded).
+        Returns (ids, n_groups[, first_row int64 tensor of the groups' smallest row])."""
+        import torch
+        dev = keys[0].data.device
+        if ids is None:
+            ids = torch.zeros(keys[0].n, dtype=torch.int32, device=dev)
+        f = torch.empty(max(keys[0].n, 1), dtype=torch.int64, device=dev) if first else None
+        ng = ctypes.c_int64(0)
+        _chk(lib().up_group_ids(self.h, _descs(keys), len(keys), ids.data_ptr(), ctypes.byref(ng),
+                                f.data_ptr() if f is not None else None, _stream_ptr(stream)))
+        return (ids, ng.value, f[:ng.value]) if first else (ids, ng.value)
 
     def check(self, stream=None):
         _chk(lib().up_check(self.h, _stream_ptr(stream)))
