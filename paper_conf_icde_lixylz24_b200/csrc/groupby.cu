@@ -17,6 +17,7 @@
 
 up_status up_internal_fail(up_status st, const std::string &msg);
 void up_internal_add_launches(up_ctx *c, long long k);
+up_status up_internal_scratch(up_ctx *c, size_t bytes, void **out);
 
 namespace {
 
@@ -104,21 +105,22 @@ extern "C" up_status up_group_ids(up_ctx *c, const up_column *keys, int nkeys, i
     *n_groups = 0;
     if (n == 0) return UP_OK;
     cudaStream_t st = (cudaStream_t)stream;
-    uint32_t *buf = nullptr;
-    // keys x2, perm x2, head, gid
-    if (cudaMallocAsync((void **)&buf, sizeof(uint32_t) * 6 * (size_t)n, st) != cudaSuccess)
-        return up_internal_fail(UP_E_NOMEM, "group_ids: scratch allocation failed");
-    uint32_t *k0 = buf, *k1 = buf + n, *p0 = buf + 2 * n, *p1 = buf + 3 * n, *head = buf + 4 * n, *gid = buf + 5 * n;
-    cub::DoubleBuffer<uint32_t> kb(k0, k1), pb(p0, p1);
+    // scratch (the ctx's persistent buffer): keys x2, perm x2, head, gid, then CUB's temp storage
+    uint32_t *k0 = nullptr;
     size_t tsort = 0, tscan = 0;
-    cub::DeviceRadixSort::SortPairs(nullptr, tsort, kb, pb, n, 0, 32, st);
-    cub::DeviceScan::InclusiveSum(nullptr, tscan, head, gid, n, st);
-    const size_t tbytes = tsort > tscan ? tsort : tscan;
-    void *temp = nullptr;
-    if (cudaMallocAsync(&temp, tbytes, st) != cudaSuccess) {
-        cudaFreeAsync(buf, st);
-        return up_internal_fail(UP_E_NOMEM, "group_ids: temp allocation failed");
+    {
+        cub::DoubleBuffer<uint32_t> kq(nullptr, nullptr), pq(nullptr, nullptr);
+        cub::DeviceRadixSort::SortPairs(nullptr, tsort, kq, pq, n, 0, 32, st);
+        cub::DeviceScan::InclusiveSum(nullptr, tscan, (uint32_t *)nullptr, (uint32_t *)nullptr, n, st);
     }
+    const size_t tbytes = tsort > tscan ? tsort : tscan;
+    const size_t words = ((6 * (size_t)n + 63) / 64) * 64;
+    void *base = nullptr;
+    if (up_status e = up_internal_scratch(c, words * sizeof(uint32_t) + tbytes, &base)) return e;
+    k0 = (uint32_t *)base;
+    void *temp = (void *)(k0 + words);
+    uint32_t *k1 = k0 + n, *p0 = k0 + 2 * n, *p1 = k0 + 3 * n, *head = k0 + 4 * n, *gid = k0 + 5 * n;
+    cub::DoubleBuffer<uint32_t> kb(k0, k1), pb(p0, p1);
     const int grid = grid_for(n);
     long long launches = 0;
     k_gb_iota<<<grid, 256, 0, st>>>(pb.Current(), n);
@@ -150,8 +152,6 @@ extern "C" up_status up_group_ids(up_ctx *c, const up_column *keys, int nkeys, i
     cudaMemcpyAsync(&total, gid + (n - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st);
     k_gb_scatter<<<grid, 256, 0, st>>>(pb.Current(), head, gid, d_ids, reinterpret_cast<long long *>(d_first), n);
     ++launches;
-    cudaFreeAsync(temp, st);
-    cudaFreeAsync(buf, st);
     up_internal_add_launches(c, launches);
     const cudaError_t e = cudaStreamSynchronize(st);
     if (e != cudaSuccess) return up_internal_fail(UP_E_CUDA, std::string("group_ids: ") + cudaGetErrorString(e));
