@@ -28,13 +28,14 @@ def test_textbook_rsa_on_gpu():
 @pytest.mark.parametrize("e", [3, 65537])
 @pytest.mark.parametrize("radix", ["r28", "r32"])
 def test_modexp_parity(bits, e, radix, monkeypatch):
-    """Both Montgomery kernels: radix 2^28 (default up to 40 32-bit limbs;
-    1034 bits puts 4N right under R = 2^1036) and the 32-bit CIOS
-    (UP_MONT32=1, and every modulus wider than 40 limbs)."""
+    """Both Montgomery kernels: radix 2^28 (default up to 64 32-bit limbs,
+    the base in shared memory beyond 40; 1034 bits puts 4N right under
+    R = 2^1036) and the 32-bit CIOS (UP_MONT32=1, and every modulus wider
+    than 64 limbs)."""
     if radix == "r32":
         monkeypatch.setenv("UP_MONT32", "1")
-    elif bits > 40 * 32:
-        pytest.skip("radix 2^28 kernel only up to 40 limbs")
+    elif bits > 64 * 32:
+        pytest.skip("radix 2^28 kernel only up to 64 limbs")
     N, p, q = synth.rsa_modulus(bits)
     n = 333
     mag, neg = synth.rsa_messages(n, N)
