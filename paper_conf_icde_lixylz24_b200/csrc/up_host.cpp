@@ -110,6 +110,7 @@ up_status fail(up_status st, const char *fmt, ...) {
 constexpr int kThreads = 256;
 constexpr int kWsSlots = 1 << 16;
 constexpr int kContractMinProducts = 100;   // row contraction only for compute-bound products
+constexpr long kSplitAutoProducts = 80 * 80;  // automatic split from this product size on
 constexpr int kWideMinLimbs = 257;  // warp-per-row only beyond this (per-thread measured faster at p <= 1000)
 
 struct JitKernel {
@@ -700,7 +701,17 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     // rest -> the fused per-thread kernel, then an exact combine (SUM is linear).
     // opt-in (UP_SPLIT=1): measured slower than the fused per-thread kernel at
     // p = 200 (7.5 vs 2.9 ms) and only 1.2x faster at p = 1000 in round 1
-    if (getenv("UP_SPLIT") && !getenv("UP_NO_SPLIT")) {
+    // row-contraction split: forced by UP_SPLIT, automatic when a top-level
+    // column product is at least kSplitAutoProducts limb products (measured on
+    // B200: cfg3 p = 1000 (104 x 104 limbs) 5.9e7 -> 7.2e7 rows/s; p = 500
+    // (52 x 52) and p = 200 stay faster fused), off with UP_NO_SPLIT
+    bool try_split = getenv("UP_SPLIT") != nullptr;
+    if (!try_split && !getenv("UP_NO_SPLIT")) {
+        for (int i = 0; i < ncols && !try_split; ++i)
+            for (int j = 0; j < ncols && !try_split; ++j)
+                if ((long)cols[i].limbs * cols[j].limbs >= kSplitAutoProducts) try_split = true;
+    }
+    if (try_split && !getenv("UP_NO_SPLIT")) {
         Typed ts;
         if (up_status s = type_expr(expr, cols, ncols, ts)) return s;
         const int LAs = limbs_for_precision(sum_precision(ts.root->p, N));
@@ -727,8 +738,14 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
                 std::string key = "contract|" + std::to_string(La) + "|" + std::to_string(Lb) + "|" + std::to_string(LAs) +
                                   "|" + std::to_string(st.sign) + "|" + std::to_string(st.col_a) + "|" + std::to_string(st.col_b);
                 JitKernel *kc = nullptr;
+                // radix-2^28 contraction: opt-in (measured: equal at p = 1000, slower at p = 500)
+                const bool r28 = getenv("UP_CONTRACT28") != nullptr;
+                if (r28) key += "|r28";
                 if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
-                        return gen_contract_kernel(La, Lb, LAs, st.sign, st.col_a, st.col_b, info); }, &kc))
+                        std::string src;
+                        if (r28) src = gen_contract_kernel28(La, Lb, LAs, st.sign, st.col_a, st.col_b, info);
+                        if (src.empty()) { info = GenInfo(); src = gen_contract_kernel(La, Lb, LAs, st.sign, st.col_a, st.col_b, info); }
+                        return src; }, &kc))
                     return s;
                 P.result = c->d_parts + (size_t)ti++ * LAs;
                 if (up_status s = launch(c, kc, P, P.n, (cudaStream_t)stream)) return s;
@@ -1013,7 +1030,8 @@ up_status up_expr_optimized(const char *expr, const up_column *cols, int ncols, 
 // generated row-contraction source (diagnostics / prewarm)
 up_status up_gen_contract_source(int32_t La, int32_t Lb, int32_t LA, int sign, char *buf, size_t len) {
     GenInfo info;
-    std::string src = gen_contract_kernel(La, Lb, LA, sign, 0, 1, info);
+    std::string src = getenv("UP_CONTRACT28") ? gen_contract_kernel28(La, Lb, LA, sign, 0, 1, info) : "";
+    if (src.empty()) { info = GenInfo(); src = gen_contract_kernel(La, Lb, LA, sign, 0, 1, info); }
     if (src.empty()) return fail(UP_E_UNSUPPORTED, "no contraction kernel");
     if (src.size() + 1 > len) return fail(UP_E_NOMEM, "buffer too small");
     memcpy(buf, src.c_str(), src.size() + 1);

@@ -85,11 +85,15 @@ def test_wide_and_per_thread_paths_agree(monkeypatch):
     ("-c1*c2 + c3*c1 - c2", [(150, 10), (150, 10), (140, 10)], ()),
     ("c1*c2 - c3/c4", [(1000, 100)] * 4, (3,)),
 ])
-def test_split_sum_matches_unsplit_and_oracle(expr, types, lead, monkeypatch):
+@pytest.mark.parametrize("radix", ["r28", "r32"])
+def test_split_sum_matches_unsplit_and_oracle(expr, types, lead, radix, monkeypatch):
     """Row-contraction SUM (products as carry-save column sums over rows, signs
-    by correction terms) + fused rest kernel + combine == oracle == UP_NO_SPLIT."""
+    by correction terms) + fused rest kernel + combine == oracle == UP_NO_SPLIT,
+    for the 32-bit contraction (default) and the radix-2^28 one (UP_CONTRACT28)."""
     n = 300 if types[0][0] >= 1000 else 2000
     monkeypatch.setenv("UP_SPLIT", "1")
+    if radix == "r28":
+        monkeypatch.setenv("UP_CONTRACT28", "1")
     host = G.gen_cols(n, types, config=3, nonzero_lead_cols=lead, seed=11)
     want, P, S = oracle.eval_sum(expr, G.to_oracle(host, types), threads=8)
     from paper_conf_icde_lixylz24_b200 import up
@@ -99,6 +103,40 @@ def test_split_sum_matches_unsplit_and_oracle(expr, types, lead, monkeypatch):
     c.check()
     assert got == want
     monkeypatch.delenv("UP_SPLIT")
+    monkeypatch.setenv("UP_NO_SPLIT", "1")
     c2 = up.Context(0)
     cols2 = [c2.column_from_host_bin(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
     assert up.result_to_string(c2.sum_expr(expr, cols2), S) == want
+
+
+@pytest.mark.parametrize("p", [200, 1000])
+@pytest.mark.parametrize("radix", ["r28", "r32"])
+def test_split_contraction_extreme_values(p, radix, monkeypatch):
+    """All-nines magnitudes (every 28-bit digit near 2^28 - 1, the column-sum
+    bound) with mixed signs over many rows per thread: SUM(c1*c2) by the
+    row contraction (both radices) == exact Python value."""
+    monkeypatch.setenv("UP_SPLIT", "1")
+    if radix == "r28":
+        monkeypatch.setenv("UP_CONTRACT28", "1")
+    import numpy as np
+    from paper_conf_icde_lixylz24_b200 import up
+    n = 5000 if p == 200 else 600
+    big = 10 ** p - 1
+    vals1 = [big if i % 3 else -big for i in range(n)]
+    vals2 = [-big if i % 5 == 0 else big for i in range(n)]
+    def words(vals):
+        w = (big.bit_length() + 31) // 32
+        mag = np.zeros((n, w), np.uint32); neg = np.zeros(n, np.uint8)
+        for i, v in enumerate(vals):
+            a = abs(v)
+            for j in range(w):
+                mag[i, j] = (a >> (32 * j)) & 0xFFFFFFFF
+            neg[i] = v < 0
+        return mag, neg
+    c = up.Context(0)
+    cols = [c.column_from_host_bin(p, 10, *words(vals1)), c.column_from_host_bin(p, 10, *words(vals2))]
+    P, S, LA = c.sum_type("c1*c2", cols)
+    got = up.result_to_string(c.sum_expr("c1*c2", cols), S)
+    c.check()
+    want = sum(a * b for a, b in zip(vals1, vals2))
+    assert got == up._fmt(want, S)
