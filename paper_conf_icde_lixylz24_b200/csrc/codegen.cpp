@@ -10,6 +10,7 @@
 #include "codegen.h"
 
 #include <cstdlib>
+#include <functional>
 #include <sstream>
 
 namespace uph {
@@ -42,10 +43,54 @@ int mag_limbs_of_pow10(int k) {   // limbs of the magnitude 10^k - 1 (at least 1
     return std::max(1, (bl + 31) / 32);
 }
 
+// Window of the top-limb division decision (div_top_decide in up_dev.cuh):
+// T divisor limbs, T = max(limbs(C), limbs(q)) + 2 so that an undecided row
+// has probability ~2^-64 for a full-length divisor; used when the divisor is
+// wider than the window and the dividend reaches into it.  Returns T, or 0.
+int div_top_window(const Node *n) {
+    if (n->op != Op::Div || getenv("UP_NO_DIVTOP")) return 0;
+    const int La = n->l->L, Lb = n->r->L;
+    const int NC = (int)HBig::pow10(n->r->s + 4).w.size();
+    const int T = std::max(NC, n->L) + 2;
+    const int E = Lb - T;
+    return (E > 0 && La > E) ? T : 0;
+}
+
+// columns read only as operands of top-limb divisions are not loaded whole:
+// those divisions read the limbs they need from global memory
+void div_only_uses(const Node *n, std::vector<int> &uses, std::vector<int> &div_uses) {
+    if (!n) return;
+    if (n->op == Op::Col) { uses[(size_t)n->col]++; return; }
+    if (div_top_window(n)) {
+        for (const Node *ch : {n->l.get(), n->r.get()}) {
+            if (ch->op == Op::Col) { uses[(size_t)ch->col]++; div_uses[(size_t)ch->col]++; }
+            else div_only_uses(ch, uses, div_uses);
+        }
+        return;
+    }
+    div_only_uses(n->l.get(), uses, div_uses);
+    div_only_uses(n->r.get(), uses, div_uses);
+}
+
 struct Emitter {
     std::ostringstream o;
     int tmp = 0;
+    std::vector<bool> lazy;   // column c is read from global memory by the divisions that use it
     std::string fresh(const char *pfx) { return std::string(pfx) + std::to_string(tmp++); }
+    bool is_lazy(const Node *n) const { return n->op == Op::Col && (size_t)n->col < lazy.size() && lazy[(size_t)n->col]; }
+    // limb j (static) of operand n: register array x, or a global load for a lazy column
+    std::string limb(const Node *n, const std::string &x, int j) const {
+        if (is_lazy(n)) return "__ldg(g" + std::to_string(n->col) + " + (long long)" + std::to_string(j) + " * l" + std::to_string(n->col) + ")";
+        return x + "[" + std::to_string(j) + "]";
+    }
+    // the whole operand as a register array (loads a lazy column)
+    std::string whole(const Node *n, const std::string &x) {
+        if (!is_lazy(n)) return x;
+        std::string t = fresh("t");
+        o << "    u32 " << t << "[" << n->L << "];\n#pragma unroll\n    for (int j = 0; j < " << n->L << "; ++j) " << t
+          << "[j] = __ldg(g" << n->col << " + (long long)j * l" << n->col << ");\n";
+        return t;
+    }
 
     // constant array of exactly `n` limbs holding v (truncated / zero padded)
     std::string konst(const HBig &v, int n) {
@@ -133,12 +178,32 @@ struct Emitter {
             const int NU = mag_limbs_of_pow10(L_->p + k);
             HBig c = HBig::pow10(k);
             std::string ua = fresh("t"), na = fresh("n"), ub = fresh("t"), nb = fresh("n"), uu = fresh("t"), rr = fresh("t");
+            std::string kc = konst(c, (int)c.w.size());
+            const int T = div_top_window(n);
+            if (T) {
+                // top-limb decision (div_top_decide), the full Knuth division only for undecided rows
+                const int E = Lb - T, NAH = La - E;
+                std::string ah = fresh("t"), vh = fresh("t");
+                // signs in {0,1} (cond_neg's contract); complement masks 0 - sign
+                o << "    u32 " << t << "[" << L << "], " << na << " = " << limb(L_, a, La - 1) << " >> 31, " << nb
+                  << " = " << limb(R_, b, Lb - 1) << " >> 31;\n";
+                o << "    u32 " << ah << "[" << NAH << "], " << vh << "[" << T << "];\n";
+                for (int j = 0; j < NAH; ++j) o << "    " << ah << "[" << j << "] = " << limb(L_, a, E + j) << " ^ (0u - " << na << ");\n";
+                for (int j = 0; j < T; ++j) o << "    " << vh << "[" << j << "] = " << limb(R_, b, E + j) << " ^ (0u - " << nb << ");\n";
+                o << "    if (!div_top_decide<" << NAH << "," << T << "," << c.w.size() << "," << L << ">(" << t << ", " << ah << ", " << vh << ", " << kc << ")) {\n";
+                const std::string fa = whole(L_, a), fb = whole(R_, b);
+                o << "    u32 " << ua << "[" << La << "], " << ub << "[" << Lb << "], " << na << "x, " << nb << "x; abs_copy(" << ua << ", " << fa << ", " << na << "x); abs_copy(" << ub << ", " << fb << ", " << nb << "x);\n";
+                o << "    u32 " << uu << "[" << NU << "]; mul_mag<" << La << "," << c.w.size() << "," << NU << ">(" << uu << ", " << ua << ", " << kc << ");\n";
+                o << "    u32 " << rr << "[" << Lb << "];\n";
+                o << "    fl |= divmod_mag<" << NU << "," << Lb << "," << L << ",false>(" << t << ", " << rr << ", " << uu << ", " << ub << ");\n";
+                o << "    }\n";
+            } else {
             o << "    u32 " << ua << "[" << La << "], " << na << "; abs_copy(" << ua << ", " << a << ", " << na << ");\n";
             o << "    u32 " << ub << "[" << Lb << "], " << nb << "; abs_copy(" << ub << ", " << b << ", " << nb << ");\n";
-            std::string kc = konst(c, (int)c.w.size());
             o << "    u32 " << uu << "[" << NU << "]; mul_mag<" << La << "," << c.w.size() << "," << NU << ">(" << uu << ", " << ua << ", " << kc << ");\n";
             o << "    u32 " << t << "[" << L << "], " << rr << "[" << Lb << "];\n";
             o << "    fl |= divmod_mag<" << NU << "," << Lb << "," << L << ",false>(" << t << ", " << rr << ", " << uu << ", " << ub << ");\n";
+            }
             // declared-type check |Q| < 10^p (reading Q5: the paper's bound can fail)
             std::string kb = konst(HBig::pow10(n->p), L);
             o << "    if (!lt(" << t << ", " << kb << ")) fl |= F_OVERFLOW;\n";
@@ -173,6 +238,12 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     info.rows_per_thread = R;
 
     Emitter E;
+    {
+        std::vector<int> uses(cols.size(), 0), div_uses(cols.size(), 0);
+        div_only_uses(root, uses, div_uses);
+        E.lazy.assign(cols.size(), false);
+        for (size_t c = 0; c < cols.size(); ++c) E.lazy[c] = used[c] && uses[c] > 0 && uses[c] == div_uses[c];
+    }
     std::string res = E.emit(root);
 
     std::ostringstream k;
@@ -183,7 +254,8 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     bool first = true;
     for (size_t c = 0; c < cols.size(); ++c) {
         if (!used[c]) continue;
-        k << (first ? "" : ", ") << "const u32 (&x" << c << ")[" << cols[c].limbs << "]";
+        if (E.lazy[c]) k << (first ? "" : ", ") << "const u32 *__restrict__ g" << c << ", long long l" << c;
+        else k << (first ? "" : ", ") << "const u32 (&x" << c << ")[" << cols[c].limbs << "]";
         first = false;
     }
     k << (first ? "" : ", ") << "u32 (&res)[" << LOUT << "], u32 &fl) {\n";
@@ -192,19 +264,29 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
 
     const bool cs = LOUT <= 8;
     const int LA = opt.sum ? opt.LA : LOUT;
-    const int NS = cs ? LOUT : LA;
-    k << "extern \"C\" __global__ void " << launch_bounds(256, (R == 1 && max_limbs(root) <= 64) ? 2 : 0) << " upk(const up_kparams P) {\n";
+    // chain accumulator: LOUT + 1 limbs per thread (< 2^31 rows per thread),
+    // its sign as a negative count at slot KC -- not LA limbs (LA can be 20x LOUT)
+    const int KC = std::min(LA, LOUT + 1);
+    const int NS = cs ? LOUT : KC;
+    // registers held across the row: node widths, minus columns only the
+    // top-limb divisions read (loaded per division, not kept)
+    std::function<int(const Node *)> live = [&](const Node *x) -> int {
+        if (!x) return 0;
+        if (E.is_lazy(x)) return 0;
+        return std::max(x->L, std::max(live(x->l.get()), live(x->r.get())));
+    };
+    k << "extern \"C\" __global__ void " << launch_bounds(256, (R == 1 && live(root) <= 64) ? 2 : 0) << " upk(const up_kparams P) {\n";
     k << "    constexpr int R = " << R << ";\n";
     k << "    u32 fl = 0;\n";
     if (opt.sum) {
         if (cs) k << "    AccCS<" << LOUT << "> acc; acc.init();\n";
-        else k << "    AccChain<" << LOUT << "," << LA << "> acc; acc.init();\n";
+        else k << "    AccChain<" << LOUT << "," << KC << "> acc; acc.init();\n";
     }
     k << "    const long long n = P.n;\n";
     k << "    const long long stride = (long long)gridDim.x * blockDim.x * R;\n";
     k << "    for (long long base = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * R; base < n; base += stride) {\n";
     for (size_t c = 0; c < cols.size(); ++c) {
-        if (!used[c]) continue;
+        if (!used[c] || E.lazy[c]) continue;
         const int Lc = cols[c].limbs;
         k << "        u32 x" << c << "[R][" << Lc << "];\n";
         k << "        { const u32 *p = P.col[" << c << "] + base; const long long ld = P.ld[" << c << "];\n";
@@ -223,7 +305,8 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     first = true;
     for (size_t c = 0; c < cols.size(); ++c) {
         if (!used[c]) continue;
-        k << (first ? "" : ", ") << "x" << c << "[r]";
+        if (E.lazy[c]) k << (first ? "" : ", ") << "P.col[" << c << "] + base + r, P.ld[" << c << "]";
+        else k << (first ? "" : ", ") << "x" << c << "[r]";
         first = false;
     }
     k << (first ? "" : ", ") << "v, fr);\n";
@@ -254,8 +337,8 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
             k << "    block_commit<" << NS << "," << LA << "," << LOUT << ">(vals, P.ws, P.ticket, P.result, sm);\n";
         } else {
             k << "#pragma unroll\n    for (int j = 0; j < " << NS << "; ++j) vals[j] = acc.a[j];\n";
-            k << "    vals[" << NS << "] = 0ull;\n";
-            k << "    block_commit<" << NS << "," << LA << "," << LA << ">(vals, P.ws, P.ticket, P.result, sm);\n";
+            k << "    vals[" << NS << "] = " << (KC < LA ? "(u64)(acc.a[" + std::to_string(KC - 1) + "] >> 31)" : std::string("0ull")) << ";\n";
+            k << "    block_commit<" << NS << "," << LA << "," << NS << ">(vals, P.ws, P.ticket, P.result, sm);\n";
         }
         info.ws_slots = NS + 1;
     }
