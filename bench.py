@@ -173,16 +173,26 @@ class ExprWorkload(Workload):
         self.ctx.sum_expr(self.cfg["expr"], self.e2e_cols, self.n_global, out=out)
 
     def roofline(self, kernel_ms, peaks):
-        if self.cfg["types"][0][0] >= 100:     # wide expressions: integer-pipe bound
+        tc = not (os.environ.get("UP_NO_TC") or os.environ.get("UP_NO_SPLIT"))
+        if self.cfg["types"][0][0] >= 100 and not tc:     # wide expressions on CUDA cores: integer-pipe bound
             return self._alu_roofline(kernel_ms, self.alg_products_per_row())
+        # HBM roofline.  Wide expressions with the tensor-core split (default):
+        # SUM(c1*c2) is an integer GEMM over the rows on tcgen05 (kind::i8,
+        # contract_tc.cu) whose FLOPs are ~1/30 of the tensor peak, c3/c4 is
+        # decided from the operands' top limbs -- what remains is moving the
+        # columns; algorithmic bytes = every limb plane of every column
         alg = self.bytes_per_row * self.rows
         peak = peaks.get("hbm_gbs", 6650.0)
         ach = alg / (kernel_ms / 1e3) / 1e9
-        return {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(ach / peak, 4), "kernel_ms": round(kernel_ms, 5), "alg_bytes_per_launch": alg,
-                "alg_unit": f"{self.bytes_per_row} B/row (limb planes read) x {self.rows} rows",
-                "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks
-                else "fallback 6.65 TB/s"}
+        r = {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
+             "frac": round(ach / peak, 4), "kernel_ms": round(kernel_ms, 5), "alg_bytes_per_launch": alg,
+             "alg_unit": f"{self.bytes_per_row} B/row (limb planes of all columns) x {self.rows} rows",
+             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks
+             else "fallback 6.65 TB/s"}
+        if self.cfg["types"][0][0] >= 100:
+            r["note"] = ("step = tensor-core row contraction SUM(c1*c2) (u8 digits, s32 TMEM accumulators) "
+                         "+ fused per-thread rest (top-limb division) + exact combine")
+        return r
 
     def alg_products_per_row(self):
         """limb products of c1*c2 - c3/c4 = x (L*L) + / prescale

@@ -1,0 +1,458 @@
+// contract_tc.cu -- SUM over rows of c_a * c_b (a top-level column product of
+// SELECT SUM(expr), SURVEY §8a rows a6 + a11) on the 5th-generation tensor
+// cores, exact.
+//
+// The SUM of a product of two DECIMAL columns is a dense contraction over the
+// row index: with byte digits a_x (x < 4La) of the two's-complement limb
+// planes of c_a, and the sign digit a_{4La} = s_a (weight -2^(32 La)),
+//     SUM_i a_i b_i = SUM_{x,y} sgn(x,y) 2^(8(x+y)) D[x][y],
+//     D[x][y] = SUM_i a_x(i) b_y(i)                    (u8 x u8 -> s32),
+// sgn = -1 when exactly one of x, y is a sign digit (schoolbook product of
+// P:L576-607 with the row sum of P:L1069-1080 moved inside it, which SUM's
+// linearity allows).  D is one integer GEMM (M = digits of c_a, N = digits
+// of c_b, K = rows) issued as tcgen05.mma kind::i8 with the accumulator in
+// TMEM.  The limb planes are not K-major byte matrices, so the CTA's threads
+// load 16-row x 1-limb pieces (4 x LDG.128), transpose bytes with PRMT and
+// write the canonical no-swizzle K-major core-matrix layout into shared
+// memory (two stages); one thread issues the MMAs and commits them to an
+// mbarrier.  Every <= 32768 rows (255^2 * 32768 < 2^31) the accumulator is
+// drained: each thread reads its TMEM lane (one digit x) and adds D[x][y]
+// into per-CTA anti-diagonal sums (u64, shared memory).  At the end the
+// CTAs add their sums into 32-bit-aligned u64 slots (positive and negative
+// parts) with global atomics and the last CTA normalises them into LA
+// two's-complement limbs: exact for any row count < 2^32.
+//
+// Roles: M tile (128 digits of c_a) x N group (<= 512 digits of c_b, the
+// TMEM width), so one CTA's accumulator fits TMEM; CTAs of the same row block
+// run the roles of the same rows (c_b re-reads hit L2).
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+namespace {
+
+typedef uint32_t u32;
+typedef unsigned long long u64;
+
+constexpr int THREADS = 256;
+constexpr int NRAW = 3;                  // raw (bulk-copied) stages in flight
+constexpr int MAX_SLOTS = 1024;
+constexpr int MAX_ROLE_LIMBS = 256;
+constexpr int ABOX = 32;                 // c_a limbs per M tile (128 digits)
+
+struct TcArgs {
+    const u32 *A, *B;
+    long long lda, ldb, n;
+    int La, Lb;
+    int n_mtiles, n_groups, n_roles, n_rblocks;
+    u64 *ws;          // 2 * nsl slots: positive, negative (zero on entry, re-zeroed)
+    u32 *ticket;
+    u32 *result;      // LA limbs
+    int LA, nsl, sign;
+    int bbox;         // c_b limbs per N group box (<= 128)
+};
+
+__device__ __forceinline__ u32 smem_u32(const void *p) { return (u32)__cvta_generic_to_shared(p); }
+
+// K-major, no swizzle: LBO = 128 B (next 16-byte K chunk), SBO = next 8-row group
+template <int SBO>
+__device__ __forceinline__ u64 umma_desc(u32 saddr) {
+    return (u64)((saddr >> 4) & 0x3FFFu) | ((u64)(128 >> 4) << 16) | ((u64)(SBO >> 4) << 32) | (1ull << 46);
+}
+
+// bounded wait: a lost completion traps (launch error) instead of hanging.
+// try_wait with a suspend-time hint parks the warp instead of spinning.
+__device__ __forceinline__ void mbar_wait(u32 mb, u32 parity) {
+    u32 ok;
+    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+                 "selp.u32 %0, 1, 0, p;\n\t}\n" : "=r"(ok) : "r"(mb), "r"(parity), "r"(1000000u) : "memory");
+    if (ok) return;
+    for (long long spins = 0;; ++spins) {
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+                     "selp.u32 %0, 1, 0, p;\n\t}\n" : "=r"(ok) : "r"(mb), "r"(parity), "r"(1000000u) : "memory");
+        if (ok) return;
+        if (spins == (1ll << 24)) {
+            printf("contract_tc: mbarrier wait timed out (block %d thread %d parity %u)\n", blockIdx.x, threadIdx.x, parity);
+            __trap();
+        }
+    }
+}
+
+// byte b of four words -> one word (b < 4), or their sign bits (b == 4)
+__device__ __forceinline__ u32 pick4(u32 x0, u32 x1, u32 x2, u32 x3, int b) {
+    if (b == 4) return (x0 >> 31) | ((x1 >> 31) << 8) | ((x2 >> 31) << 16) | ((x3 >> 31) << 24);
+    const u32 sel = (u32)b | ((u32)(4 + b) << 4);
+    return __byte_perm(__byte_perm(x0, x1, sel), __byte_perm(x2, x3, sel), 0x5410);
+}
+
+// A role's operand tile: digits [dbase, dbase + extent) of one column; its raw
+// stage holds the limbs lo .. lo + nl - 1 (+ the top limb when only the sign
+// digit falls into the tile)
+struct Opnd {
+    int dbase, L, lo, nl, raw_off;   // raw_off: first raw slot (limbs)
+    bool extra_top;                  // raw slot nl holds limb L - 1
+    int ndig;                        // digits to write: [0, ndig) local
+};
+
+template <int KC>
+__global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P, const __grid_constant__ CUtensorMap tA,
+                                                                  const __grid_constant__ CUtensorMap tB) {
+    constexpr int NRG = KC / 16;             // 16-row groups per stage
+    constexpr int SBO = NRG * 128;           // bytes between 8-digit core-matrix groups
+    constexpr int DRAIN_CHUNKS = 32768 / KC; // s32 accumulators drained every 32768 rows
+    extern __shared__ __align__(1024) unsigned char smem[];
+    __shared__ u32 s_taddr;
+    __shared__ __align__(8) u64 s_full[NRAW], s_empty[NRAW], s_cfull[2], s_mdone[2], s_drained;
+    __shared__ u32 s_last;
+
+    // warps 0-7 transform raw limb rows into the MMA layout (warps 0-3 also
+    // drain TMEM lanes 0-127); warp 8 issues the bulk copies and the MMAs
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int role = blockIdx.x % P.n_roles, rblock = blockIdx.x / P.n_roles;
+    const int mt = role % P.n_mtiles, grp = role / P.n_mtiles;
+    const int MA = 4 * P.La + 1, MB = 4 * P.Lb + 1;
+    const int x0 = 128 * mt, y0 = 512 * grp;               // first digits of this role
+    const int ny = min(512, MB - y0);
+    const int W = (ny + 15) & ~15;                         // MMA N extent (<= 512)
+    const int N0 = W > 256 ? 256 : W, N1 = W - N0;         // two N tiles at most
+    const u32 tcols = W <= 32 ? 32 : W <= 64 ? 64 : W <= 128 ? 128 : W <= 256 ? 256 : 512;
+
+    // raw stage = TMA boxes [ABOX limbs | P.bbox limbs] x KC rows (rows >= n and
+    // limbs >= L arrive zero-filled); a box starts one limb early when only the
+    // sign digit of its column falls into the tile (it needs the top limb)
+    Opnd oa, ob;
+    oa.dbase = x0; oa.L = P.La; oa.lo = x0 / 4; oa.nl = max(0, min(P.La, (x0 + 128) / 4) - oa.lo);
+    oa.extra_top = (4 * P.La >= x0 && 4 * P.La < x0 + 128) && oa.nl == 0;
+    oa.ndig = min(128, MA - x0);
+    oa.raw_off = 0;
+    ob.dbase = y0; ob.L = P.Lb; ob.lo = y0 / 4; ob.nl = max(0, min(P.Lb, (y0 + W) / 4) - ob.lo);
+    ob.extra_top = (4 * P.Lb >= y0 && 4 * P.Lb < y0 + W) && ob.nl == 0;
+    ob.ndig = ny;
+    ob.raw_off = ABOX;
+    const int box_a = oa.extra_top ? P.La - 1 : oa.lo, box_b = ob.extra_top ? P.Lb - 1 : ob.lo;
+    const int nraw_limbs = ABOX + P.bbox;
+
+    // shared: [NRAW raw stages: limb x KC words][2 canonical stages: A 128 x KC | B W x KC][digit sums]
+    const int raw_bytes = nraw_limbs * KC * 4;
+    const int a_bytes = 128 * KC, b_bytes = W * KC, st_bytes = a_bytes + b_bytes;
+    unsigned char *raw0 = smem;
+    unsigned char *canon0 = smem + NRAW * raw_bytes;
+    const int ND = 128 + W;
+    u64 *dpos = reinterpret_cast<u64 *>(canon0 + 2 * st_bytes);
+    u64 *dneg = dpos + ND;
+
+    for (int i = tid; i < (2 * st_bytes) / 16; i += blockDim.x) reinterpret_cast<uint4 *>(canon0)[i] = make_uint4(0, 0, 0, 0);
+    for (int i = tid; i < 2 * ND; i += blockDim.x) dpos[i] = 0ull;
+    __syncwarp();
+    if (warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" :: "r"(smem_u32(&s_taddr)), "r"(tcols));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (tid == 0) {
+        for (int i = 0; i < NRAW; ++i) {
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&s_full[i])));
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;" :: "r"(smem_u32(&s_empty[i])));
+        }
+        for (int i = 0; i < 2; ++i) {
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;" :: "r"(smem_u32(&s_cfull[i])));
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&s_mdone[i])));
+        }
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 4;" :: "r"(smem_u32(&s_drained)));
+        asm volatile("fence.mbarrier_init.release.cluster;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;");
+    const u32 taddr = s_taddr;
+
+    const long long n = P.n;
+    const long long nchunks = (n + KC - 1) / KC;
+    const long long my_chunks = rblock < nchunks ? (nchunks - 1 - rblock) / P.n_rblocks + 1 : 0;
+    auto is_drain = [&](long long t) { return ((t + 1) % DRAIN_CHUNKS) == 0 || t == my_chunks - 1; };
+
+    if (warp == 8) {
+        // ---------------- control warp: bulk copies + MMA issue
+        auto issue = [&](long long t) {   // the role's limb rows of local chunk t -> raw stage t % NRAW (2 TMA boxes)
+            if (lane != 0) return;
+            const int rs = (int)(t % NRAW);
+            const int row0 = (int)((rblock + t * P.n_rblocks) * KC);
+            const u32 mb = smem_u32(&s_full[rs]);
+            const u32 tx = (u32)(nraw_limbs * KC * 4);
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(mb), "r"(tx) : "memory");
+            const u32 dst = smem_u32(raw0 + rs * raw_bytes);
+            asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                         :: "r"(dst), "l"(&tA), "r"(row0), "r"(box_a), "r"(mb) : "memory");
+            asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                         :: "r"(dst + (u32)(ABOX * KC * 4)), "l"(&tB), "r"(row0), "r"(box_b), "r"(mb) : "memory");
+        };
+        for (long long t = 0; t < NRAW && t < my_chunks; ++t) issue(t);
+        const u32 idesc0 = (2u << 4) | ((u32)(N0 >> 3) << 17) | ((128u >> 4) << 24);
+        const u32 idesc1 = (2u << 4) | ((u32)(N1 >> 3) << 17) | ((128u >> 4) << 24);
+        int drains = 0;
+        for (long long t = 0; t < my_chunks; ++t) {
+            const int cs = (int)(t & 1), rs = (int)(t % NRAW);
+            if (lane == 0) {
+                mbar_wait(smem_u32(&s_cfull[cs]), (u32)((t >> 1) & 1));           // canonical stage written
+                const bool fresh = (t == 0) || is_drain(t - 1);
+                if (t > 0 && is_drain(t - 1)) mbar_wait(smem_u32(&s_drained), (u32)(drains++ & 1));   // TMEM read out
+                asm volatile("tcgen05.fence::after_thread_sync;");
+                const u32 a_addr = smem_u32(canon0 + cs * st_bytes), b_addr = a_addr + (u32)a_bytes;
+#pragma unroll
+                for (int kk = 0; kk < KC / 32; ++kk) {
+                    const u32 acc = (!fresh || kk > 0) ? 1u : 0u;
+                    const u64 da = umma_desc<SBO>(a_addr + kk * 256);
+                    const u64 db0 = umma_desc<SBO>(b_addr + kk * 256);
+                    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                                 "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}\n"
+                                 :: "r"(taddr), "l"(da), "l"(db0), "r"(idesc0), "r"(acc));
+                    if (N1 > 0) {
+                        const u64 db1 = umma_desc<SBO>(b_addr + (N0 / 8) * SBO + kk * 256);
+                        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                                     "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}\n"
+                                     :: "r"(taddr + (u32)N0), "l"(da), "l"(db1), "r"(idesc1), "r"(acc));
+                    }
+                }
+                asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                             :: "r"(smem_u32(&s_mdone[cs])));
+                if (t + NRAW < my_chunks) mbar_wait(smem_u32(&s_empty[rs]), (u32)((t / NRAW) & 1));   // raw stage read
+            }
+            __syncwarp();
+            if (t + NRAW < my_chunks) issue(t + NRAW);
+        }
+    } else {
+        // ---------------- transform warps: per-thread task list fixed for the whole run
+        constexpr int MAXT = 16;
+        const int sub = tid & 7, quarter = tid >> 3;      // 32 quarters, 8 lanes (digits) each
+        const int ga = (oa.ndig + 7) / 8, gb = (ob.ndig + 7) / 8;
+        const int tasks = (ga + gb) * NRG;
+        u32 t_src[MAXT], t_dst[MAXT];                      // raw word offset; canonical byte offset | b << 20 | rg << 24
+        int nt = 0;
+#pragma unroll
+        for (int k = 0; k < MAXT; ++k) {
+            t_src[k] = 0; t_dst[k] = 0xFFFFFFFFu;
+            const int task = quarter + 32 * k;
+            if (task >= tasks) continue;
+            nt = k + 1;
+            const int g = task / NRG, rg = task % NRG;
+            const bool isA = g < ga;
+            const Opnd &o = isA ? oa : ob;
+            const int dl = 8 * (isA ? g : g - ga) + sub;
+            if (dl >= o.ndig) continue;
+            const int d = o.dbase + dl;
+            const int blo = isA ? box_a : box_b;
+            int sgn, slot;
+            if (d < 4 * o.L) { sgn = 0; slot = d / 4 - blo; }         // byte d & 3 == sub & 3 (tiles start at multiples of 4)
+            else if (d == 4 * o.L) { sgn = 1; slot = o.L - 1 - blo; }
+            else continue;
+            t_src[k] = (u32)((o.raw_off + slot) * KC + 16 * rg);
+            t_dst[k] = (u32)((isA ? 0 : a_bytes) + (dl >> 3) * SBO + rg * 128 + (dl & 7) * 16) | ((u32)sgn << 20);
+        }
+        const u32 sel = (u32)(sub & 3) | ((u32)(4 + (sub & 3)) << 4);   // this lane's byte of every word
+        for (long long t = 0; t < my_chunks; ++t) {
+            const int rs = (int)(t % NRAW), cs = (int)(t & 1);
+            mbar_wait(smem_u32(&s_full[rs]), (u32)((t / NRAW) & 1));               // raw rows landed
+            if (t >= 2) mbar_wait(smem_u32(&s_mdone[cs]), (u32)(((t - 2) >> 1) & 1));  // canonical stage free
+            const u32 *raw = reinterpret_cast<const u32 *>(raw0 + rs * raw_bytes);
+            unsigned char *canon = canon0 + cs * st_bytes;
+#pragma unroll
+            for (int k = 0; k < MAXT; ++k) {
+                if (k >= nt) break;
+                const u32 td = t_dst[k];
+                if (td == 0xFFFFFFFFu) continue;
+                const uint4 *src = reinterpret_cast<const uint4 *>(raw + t_src[k]);
+                uint4 w[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) w[q] = src[q];
+                uint4 out;
+                if (!(td >> 20)) {
+                    out.x = __byte_perm(__byte_perm(w[0].x, w[0].y, sel), __byte_perm(w[0].z, w[0].w, sel), 0x5410);
+                    out.y = __byte_perm(__byte_perm(w[1].x, w[1].y, sel), __byte_perm(w[1].z, w[1].w, sel), 0x5410);
+                    out.z = __byte_perm(__byte_perm(w[2].x, w[2].y, sel), __byte_perm(w[2].z, w[2].w, sel), 0x5410);
+                    out.w = __byte_perm(__byte_perm(w[3].x, w[3].y, sel), __byte_perm(w[3].z, w[3].w, sel), 0x5410);
+                } else {                                   // sign digit: top bit of the top limb
+                    out.x = pick4(w[0].x, w[0].y, w[0].z, w[0].w, 4);
+                    out.y = pick4(w[1].x, w[1].y, w[1].z, w[1].w, 4);
+                    out.z = pick4(w[2].x, w[2].y, w[2].z, w[2].w, 4);
+                    out.w = pick4(w[3].x, w[3].y, w[3].z, w[3].w, 4);
+                }
+                *reinterpret_cast<uint4 *>(canon + (td & 0xFFFFFu)) = out;
+            }
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            __syncwarp();
+            if (lane == 0) {
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(&s_empty[rs])) : "memory");
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(&s_cfull[cs])) : "memory");
+            }
+            if (warp < 4 && is_drain(t)) {
+                // accumulator drain: MMAs of chunk t done -> D[x][y] into the digit sums
+                mbar_wait(smem_u32(&s_mdone[cs]), (u32)((t >> 1) & 1));
+                asm volatile("tcgen05.fence::after_thread_sync;");
+                const int x = x0 + 32 * warp + lane;       // this thread's digit of c_a (TMEM lane)
+                const bool xs = (x == 4 * P.La), xv = x < MA;
+                for (int c0 = 0; c0 < W; c0 += 32) {
+                    u32 v[32];
+                    const u32 ta = taddr + ((u32)(32 * warp) << 16) + (u32)c0;
+                    asm volatile(
+                        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+                        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+                        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),
+                          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+                          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+                        : "r"(ta));
+                    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+                    if (xv) {
+#pragma unroll
+                        for (int k = 0; k < 32; ++k) {
+                            const int y = y0 + c0 + k;
+                            if (y < MB && v[k]) {
+                                const bool neg = xs != (y == 4 * P.Lb);
+                                atomicAdd(&(neg ? dneg : dpos)[x - x0 + y - y0], (u64)v[k]);
+                            }
+                        }
+                    }
+                }
+                asm volatile("tcgen05.fence::before_thread_sync;");
+                __syncwarp();
+                if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(&s_drained)) : "memory");
+            }
+        }
+    }
+    __syncthreads();
+
+    // per-CTA digit sums -> 32-bit-aligned u64 slots (value v at byte position d
+    // is v * 2^(8(d%4)) at slot d/4: three 32-bit pieces)
+    u64 *wpos = P.ws, *wneg = P.ws + P.nsl;
+    for (int i = tid; i < 2 * ND; i += blockDim.x) {
+        const bool ng = i >= ND;
+        const int dd = ng ? i - ND : i;
+        const u64 v = (ng ? dneg : dpos)[dd];
+        if (!v) continue;
+        const int d = x0 + y0 + dd, sl = d >> 2, r = 8 * (d & 3);
+        const u32 p0 = (u32)(v << r);
+        const u32 p1 = r ? (u32)(v >> (32 - r)) : (u32)(v >> 32);
+        const u32 p2 = r ? (u32)(v >> (64 - r)) : 0u;
+        u64 *dst = ng ? wneg : wpos;
+        if (p0 && sl < P.nsl) atomicAdd(&dst[sl], (u64)p0);
+        if (p1 && sl + 1 < P.nsl) atomicAdd(&dst[sl + 1], (u64)p1);
+        if (p2 && sl + 2 < P.nsl) atomicAdd(&dst[sl + 2], (u64)p2);
+    }
+    __threadfence();
+    __syncthreads();
+    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(taddr), "r"(tcols));
+    if (tid == 0) s_last = (atomicAdd(P.ticket, 1u) == gridDim.x - 1) ? 1u : 0u;
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    u64 *sp = reinterpret_cast<u64 *>(smem), *sn = sp + P.nsl;    // reuse shared memory (nsl <= MAX_SLOTS)
+    for (int i = tid; i < P.nsl; i += blockDim.x) { sp[i] = atomicExch(&wpos[i], 0ull); sn[i] = atomicExch(&wneg[i], 0ull); }
+    __syncthreads();
+    if (tid == 0) {
+        *P.ticket = 0u;
+        u64 cp = 0, cn = 0;
+        u32 borrow = 0, cneg = P.sign < 0 ? 1u : 0u;
+        for (int j = 0; j < P.LA; ++j) {
+            u64 tp = cp, tn = cn;
+            if (j < P.nsl) { tp += (u32)sp[j]; tn += (u32)sn[j]; }
+            if (j >= 1 && j - 1 < P.nsl) { tp += sp[j - 1] >> 32; tn += sn[j - 1] >> 32; }
+            cp = tp >> 32; cn = tn >> 32;
+            const u64 d = (u64)(u32)tp - (u32)tn - borrow;
+            borrow = (u32)(d >> 63);
+            if (P.sign < 0) {
+                const u64 g = (u64)(~(u32)d) + cneg;
+                cneg = (u32)(g >> 32);
+                P.result[j] = (u32)g;
+            } else {
+                P.result[j] = (u32)d;
+            }
+        }
+    }
+}
+
+typedef CUresult (*EncodeTiled)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+// 2-D map of a column's limb planes: dim 0 = rows (n, contiguous), dim 1 = limbs (stride ld words)
+cudaError_t make_tmap(CUtensorMap *m, const u32 *data, long long n, int L, long long ld, int box_rows, int box_limbs) {
+    static EncodeTiled enc = nullptr;
+    if (!enc) {
+        cudaDriverEntryPointQueryResult q;
+        cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void **)&enc, cudaEnableDefault, &q);
+        if (e != cudaSuccess) return e;
+        if (q != cudaDriverEntryPointSuccess || !enc) return cudaErrorSymbolNotFound;
+    }
+    const cuuint64_t dims[2] = {(cuuint64_t)(n > 0 ? n : 1), (cuuint64_t)L};
+    const cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
+    const cuuint32_t box[2] = {(cuuint32_t)box_rows, (cuuint32_t)box_limbs};
+    const cuuint32_t es[2] = {1, 1};
+    const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, (void *)data, dims, strides, box, es,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
+template <int KC>
+cudaError_t launch_kc(TcArgs P, int W, int nraw_limbs, int num_sms, cudaStream_t st) {
+    CUtensorMap tA, tB;
+    cudaError_t e0 = make_tmap(&tA, P.A, P.n, P.La, P.lda, KC, ABOX);
+    if (e0 != cudaSuccess) return e0;
+    e0 = make_tmap(&tB, P.B, P.n, P.Lb, P.ldb, KC, P.bbox);
+    if (e0 != cudaSuccess) return e0;
+    const size_t sums = sizeof(u64) * (size_t)(2 * (128 + W));
+    size_t smem = (size_t)NRAW * nraw_limbs * KC * 4 + 2 * (size_t)(128 + W) * KC + sums;
+    if (smem < sizeof(u64) * 2 * (size_t)P.nsl) smem = sizeof(u64) * 2 * (size_t)P.nsl;
+    cudaError_t e = cudaFuncSetAttribute(k_contract_tc<KC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const int tcols = W <= 32 ? 32 : W <= 64 ? 64 : W <= 128 ? 128 : W <= 256 ? 256 : 512;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_contract_tc<KC>, THREADS + 32, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+    if (per_sm > 512 / tcols) per_sm = 512 / tcols;      // TMEM columns per SM
+    if (per_sm > 2) per_sm = 2;
+    const long long nchunks = (P.n + KC - 1) / KC;
+    long long rb = ((long long)num_sms * per_sm) / P.n_roles;
+    if (rb < 1) rb = 1;
+    if (rb > nchunks) rb = nchunks > 0 ? nchunks : 1;
+    if (const char *f = getenv("UP_TC_RBLOCKS")) rb = atoll(f) > 0 ? atoll(f) : rb;   // tests: force mid-run drains
+    P.n_rblocks = (int)rb;
+    k_contract_tc<KC><<<(unsigned)(rb * P.n_roles), THREADS + 32, smem, st>>>(P, tA, tB);
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+extern "C" {
+
+// Slots of the global workspace the kernel needs (2 * nsl), for the caller's check.
+int upk_contract_tc_slots(int La, int Lb) { return 2 * (La + Lb + 3); }
+
+// SUM_rows(sign * c_a * c_b) into `result` (LA limbs, two's complement).
+// ws: >= upk_contract_tc_slots u64, zero on entry (left zero); ticket zero.
+cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, const uint32_t *B, long long ldb, int Lb,
+                                   long long n, int sign, unsigned long long *ws, uint32_t *ticket, uint32_t *result,
+                                   int LA, int num_sms, cudaStream_t st) {
+    TcArgs P;
+    P.A = A; P.B = B; P.lda = lda; P.ldb = ldb; P.n = n; P.La = La; P.Lb = Lb;
+    const int MA = 4 * La + 1, MB = 4 * Lb + 1;
+    P.n_mtiles = (MA + 127) / 128;
+    P.n_groups = (MB + 511) / 512;
+    P.n_roles = P.n_mtiles * P.n_groups;
+    P.ws = ws; P.ticket = ticket; P.result = result; P.LA = LA; P.nsl = La + Lb + 3; P.sign = sign;
+    if (P.nsl > MAX_SLOTS) return cudaErrorInvalidValue;
+    const int W = ((MB < 512 ? MB : 512) + 15) & ~15;
+    P.bbox = (W / 4 < Lb ? W / 4 : Lb) + 1;               // group limbs (+1: a sign-only tile starts one limb early)
+    if (P.bbox > 128 + 1) P.bbox = 129;
+    const int nraw = ABOX + P.bbox;
+    if (nraw > MAX_ROLE_LIMBS) return cudaErrorInvalidValue;
+    // stage depth: 128 rows when the role's raw + canonical stages fit, else 64
+    const size_t need128 = (size_t)NRAW * nraw * 128 * 4 + 2 * (size_t)(128 + W) * 128;
+    const int max_tasks = (16 + (W + 7) / 8) * (128 / 16);   // transform tasks per 128-row stage (<= 32 x MAXT)
+    if (need128 + 16 * 1024 <= 220 * 1024 && max_tasks <= 512) return launch_kc<128>(P, W, nraw, num_sms, st);
+    return launch_kc<64>(P, W, nraw, num_sms, st);
+}
+
+}  // extern "C"

@@ -9,6 +9,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <string>
+#include <mutex>
 #include <vector>
 
 namespace uph {
@@ -101,10 +102,15 @@ struct HBig {
         for (size_t i = w.size(); i-- > 0;) { uint64_t t = (r << 32) | w[i]; q.w[i] = (uint32_t)(t / d); r = t % d; }
         q.trim(); rem = (uint32_t)r; return q;
     }
+    // 10^k, memoised (typing and codegen ask for the same powers on every call;
+    // recomputing 10^2000 digit by digit costs milliseconds of host time)
     static HBig pow10(int k) {
-        HBig r(1);
-        for (int i = 0; i < k; ++i) r = r.mul_small(10);
-        return r;
+        static std::mutex mu;
+        static std::vector<HBig> memo;
+        std::lock_guard<std::mutex> g(mu);
+        if (memo.empty()) memo.push_back(HBig(1));
+        while ((int)memo.size() <= k) memo.push_back(memo.back().mul_small(10));
+        return memo[(size_t)k];
     }
     // parse decimal digits (no sign, no point); returns false on a bad char
     static bool from_dec(const std::string &s, HBig &out) {

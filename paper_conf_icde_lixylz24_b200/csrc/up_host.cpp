@@ -37,6 +37,10 @@ cudaError_t upk_launch_from_bin(const uint32_t *mag, int W, const uint8_t *neg, 
 cudaError_t upk_launch_to_bin(const uint32_t *planes, int L, long long ld, long long n, uint32_t *mag, uint8_t *neg,
                               cudaStream_t st);
 cudaError_t upk_launch_combine(const uint32_t *partials, int nranks, int la, uint32_t *out, cudaStream_t st);
+int upk_contract_tc_slots(int La, int Lb);
+cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, const uint32_t *B, long long ldb, int Lb,
+                                   long long n, int sign, unsigned long long *ws, uint32_t *ticket, uint32_t *result,
+                                   int LA, int num_sms, cudaStream_t st);
 cudaError_t upk_launch_from_compact(const uint8_t *bytes, int Lb, long long n, const uint32_t *bound, int L,
                                    uint32_t *out, long long ld, uint32_t *flags, cudaStream_t st);
 cudaError_t upk_launch_to_compact(const uint32_t *planes, int L, long long ld, long long n, uint8_t *bytes, int Lb,
@@ -127,6 +131,16 @@ struct JitKernel {
 
 }  // namespace
 
+// a split SELECT SUM: top-level column products (tensor-core or CUDA-core
+// contraction kernels) + the rest (fused per-thread kernel) + exact combine
+struct SplitPlan {
+    bool split = false;
+    int LAs = 0;
+    std::vector<uph::SplitTerm> prods;
+    std::vector<JitKernel *> cc_kernels;   // per product: CUDA-core kernel, nullptr = tensor cores
+    JitKernel *rest_kernel = nullptr;
+};
+
 struct up_ctx {
     int device = 0;
     int num_sms = 148;
@@ -142,6 +156,7 @@ struct up_ctx {
     std::map<int, uint32_t *> pow10_dev;  // 10^p magnitude in up_limbs(p) limbs
     std::unordered_map<std::string, std::unique_ptr<JitKernel>> by_src;
     std::unordered_map<std::string, JitKernel *> by_key;
+    std::unordered_map<std::string, SplitPlan> plans;   // split SUM plans (up_sum_expr)
     uint64_t launches = 0;
     double jit_ms = 0.0;
     std::mutex mu;
@@ -705,22 +720,70 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     // column product is at least kSplitAutoProducts limb products (measured on
     // B200: cfg3 p = 1000 (104 x 104 limbs) 5.9e7 -> 7.2e7 rows/s; p = 500
     // (52 x 52) and p = 200 stay faster fused), off with UP_NO_SPLIT
+    // With the tensor-core contraction (contract_tc.cu, default; UP_NO_TC for
+    // the CUDA-core one) every top-level column product of >= kContractMinProducts
+    // limb products is split off.
+    const bool use_tc = getenv("UP_NO_TC") == nullptr;
     bool try_split = getenv("UP_SPLIT") != nullptr;
     if (!try_split && !getenv("UP_NO_SPLIT")) {
+        const long thr = use_tc ? kContractMinProducts : kSplitAutoProducts;
         for (int i = 0; i < ncols && !try_split; ++i)
             for (int j = 0; j < ncols && !try_split; ++j)
-                if ((long)cols[i].limbs * cols[j].limbs >= kSplitAutoProducts) try_split = true;
+                if ((long)cols[i].limbs * cols[j].limbs >= thr) try_split = true;
     }
     if (try_split && !getenv("UP_NO_SPLIT")) {
-        Typed ts;
-        if (up_status s = type_expr(expr, cols, ncols, ts)) return s;
-        const int LAs = limbs_for_precision(sum_precision(ts.root->p, N));
-        std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(ts.root.get(), ts.types);
-        const Node *base = opt_root ? opt_root.get() : ts.root.get();
-        std::vector<SplitTerm> prods;
-        std::unique_ptr<Node> rest;
-        if (LAs <= 512 && split_sum_terms(base, ts.types, kContractMinProducts, prods, rest)) {
-            const int T = (int)prods.size() + (rest ? 1 : 0);
+        // the split plan (terms, kernels) is cached per (expression, column types, N, knobs):
+        // typing, optimising and splitting cost host time on every call otherwise
+        const bool r28 = getenv("UP_CONTRACT28") != nullptr;
+        std::string pkey = key_of("splitplan", expr, cols, ncols, 0) + "|" + std::to_string(N) + (use_tc ? "|tc" : "") +
+                           (r28 ? "|r28" : "");
+        auto pit = c->plans.find(pkey);
+        if (pit == c->plans.end()) {
+            SplitPlan pl;
+            Typed ts;
+            if (up_status s = type_expr(expr, cols, ncols, ts)) return s;
+            pl.LAs = limbs_for_precision(sum_precision(ts.root->p, N));
+            std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(ts.root.get(), ts.types);
+            const Node *base = opt_root ? opt_root.get() : ts.root.get();
+            std::unique_ptr<Node> rest;
+            pl.split = pl.LAs <= 512 && split_sum_terms(base, ts.types, kContractMinProducts, pl.prods, rest);
+            if (pl.split) {
+                const int LAs = pl.LAs;
+                for (const SplitTerm &st : pl.prods) {
+                    const int La = cols[st.col_a].limbs, Lb = cols[st.col_b].limbs;
+                    JitKernel *kc = nullptr;
+                    if (!(use_tc && upk_contract_tc_slots(La, Lb) <= kWsSlots)) {
+                        std::string key = "contract|" + std::to_string(La) + "|" + std::to_string(Lb) + "|" + std::to_string(LAs) +
+                                          "|" + std::to_string(st.sign) + "|" + std::to_string(st.col_a) + "|" + std::to_string(st.col_b);
+                        // radix-2^28 contraction: opt-in (measured: equal at p = 1000, slower at p = 500)
+                        if (r28) key += "|r28";
+                        if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
+                                std::string src;
+                                if (r28) src = gen_contract_kernel28(La, Lb, LAs, st.sign, st.col_a, st.col_b, info);
+                                if (src.empty()) { info = GenInfo(); src = gen_contract_kernel(La, Lb, LAs, st.sign, st.col_a, st.col_b, info); }
+                                return src; }, &kc))
+                            return s;
+                    }
+                    pl.cc_kernels.push_back(kc);   // nullptr: tensor-core contraction
+                }
+                if (rest) {
+                    std::string key = "rest|" + canonical(rest.get()) + "|" + std::to_string(LAs);
+                    for (int i = 0; i < ncols; ++i) key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
+                    Node *rr = rest.get();
+                    if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
+                            GenOpts o;
+                            o.sum = true;
+                            o.LA = LAs;
+                            return gen_expr_kernel(rr, ts.types, o, info); }, &pl.rest_kernel))
+                        return s;
+                }
+            }
+            pit = c->plans.emplace(pkey, std::move(pl)).first;
+        }
+        const SplitPlan &pl = pit->second;
+        if (pl.split) {
+            const int LAs = pl.LAs;
+            const int T = (int)pl.prods.size() + (pl.rest_kernel ? 1 : 0);
             const size_t need = (size_t)T * (size_t)LAs;
             if (need > c->parts_words) {
                 if (c->d_parts) { CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream)); CUDA_TRY(cudaFree(c->d_parts)); }
@@ -733,36 +796,22 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             P.ticket = c->d_ticket;
             P.flags = c->d_flags;
             int ti = 0;
-            for (const SplitTerm &st : prods) {
-                const int La = cols[st.col_a].limbs, Lb = cols[st.col_b].limbs;
-                std::string key = "contract|" + std::to_string(La) + "|" + std::to_string(Lb) + "|" + std::to_string(LAs) +
-                                  "|" + std::to_string(st.sign) + "|" + std::to_string(st.col_a) + "|" + std::to_string(st.col_b);
-                JitKernel *kc = nullptr;
-                // radix-2^28 contraction: opt-in (measured: equal at p = 1000, slower at p = 500)
-                const bool r28 = getenv("UP_CONTRACT28") != nullptr;
-                if (r28) key += "|r28";
-                if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
-                        std::string src;
-                        if (r28) src = gen_contract_kernel28(La, Lb, LAs, st.sign, st.col_a, st.col_b, info);
-                        if (src.empty()) { info = GenInfo(); src = gen_contract_kernel(La, Lb, LAs, st.sign, st.col_a, st.col_b, info); }
-                        return src; }, &kc))
-                    return s;
+            for (size_t q = 0; q < pl.prods.size(); ++q) {
+                const SplitTerm &st = pl.prods[q];
+                const up_column &ca = cols[st.col_a], &cb = cols[st.col_b];
+                if (!pl.cc_kernels[q]) {
+                    CUDA_TRY(upk_launch_contract_tc(ca.data, ca.ld, ca.limbs, cb.data, cb.ld, cb.limbs, cols[0].n, st.sign,
+                                                    c->d_ws, c->d_ticket, c->d_parts + (size_t)ti++ * LAs, LAs, c->num_sms,
+                                                    (cudaStream_t)stream));
+                    c->launches++;
+                    continue;
+                }
                 P.result = c->d_parts + (size_t)ti++ * LAs;
-                if (up_status s = launch(c, kc, P, P.n, (cudaStream_t)stream)) return s;
+                if (up_status s = launch(c, pl.cc_kernels[q], P, P.n, (cudaStream_t)stream)) return s;
             }
-            if (rest) {
-                std::string key = "rest|" + canonical(rest.get()) + "|" + std::to_string(LAs);
-                for (int i = 0; i < ncols; ++i) key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
-                JitKernel *kr = nullptr;
-                Node *rr = rest.get();
-                if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
-                        GenOpts o;
-                        o.sum = true;
-                        o.LA = LAs;
-                        return gen_expr_kernel(rr, ts.types, o, info); }, &kr))
-                    return s;
+            if (pl.rest_kernel) {
                 P.result = c->d_parts + (size_t)ti++ * LAs;
-                if (up_status s = launch(c, kr, P, P.n, (cudaStream_t)stream)) return s;
+                if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream)) return s;
             }
             CUDA_TRY(upk_launch_combine(c->d_parts, T, LAs, d_partial, (cudaStream_t)stream));
             c->launches++;
