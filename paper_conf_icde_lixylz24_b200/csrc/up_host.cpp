@@ -157,6 +157,12 @@ struct up_ctx {
     std::unordered_map<std::string, std::unique_ptr<JitKernel>> by_src;
     std::unordered_map<std::string, JitKernel *> by_key;
     std::unordered_map<std::string, SplitPlan> plans;   // split SUM plans (up_sum_expr)
+    // side stream of a split SUM: the (ALU-bound) rest kernel overlaps the
+    // (HBM-bound) tensor-core contraction; it has its own SUM workspace
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    unsigned long long *d_ws2 = nullptr;
+    uint32_t *d_ticket2 = nullptr;
     uint64_t launches = 0;
     double jit_ms = 0.0;
     std::mutex mu;
@@ -471,6 +477,11 @@ up_status up_ctx_destroy(up_ctx *c) {
     if (c->d_stage) cudaFree(c->d_stage);
     if (c->d_scratch) cudaFree(c->d_scratch);
     if (c->d_parts) cudaFree(c->d_parts);
+    if (c->d_ws2) cudaFree(c->d_ws2);
+    if (c->d_ticket2) cudaFree(c->d_ticket2);
+    if (c->side) cudaStreamDestroy(c->side);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
     delete c;
     return UP_OK;
 }
@@ -796,6 +807,15 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             P.ticket = c->d_ticket;
             P.flags = c->d_flags;
             int ti = 0;
+            // the rest kernel runs on the side stream, concurrently with the contractions
+            // opt-in (UP_OVERLAP=1): measured slower on B200 (cfg3 p=200 1.42 -> 2.09 ms): one rest
+            // block per SM beside the contraction's CTA is slower than the two kernels back to back
+            const bool overlap = pl.rest_kernel && !pl.prods.empty() && getenv("UP_OVERLAP");
+            if (overlap && c->side) {
+                // fork before the contractions are enqueued: the side stream waits only for earlier work
+                CUDA_TRY(cudaEventRecord(c->ev_fork, (cudaStream_t)stream));
+                CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+            }
             for (size_t q = 0; q < pl.prods.size(); ++q) {
                 const SplitTerm &st = pl.prods[q];
                 const up_column &ca = cols[st.col_a], &cb = cols[st.col_b];
@@ -809,10 +829,36 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
                 P.result = c->d_parts + (size_t)ti++ * LAs;
                 if (up_status s = launch(c, pl.cc_kernels[q], P, P.n, (cudaStream_t)stream)) return s;
             }
-            if (pl.rest_kernel) {
+            if (overlap) {
+                if (!c->side) {
+                    CUDA_TRY(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
+                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+                    CUDA_TRY(cudaMalloc(&c->d_ws2, sizeof(unsigned long long) * kWsSlots));
+                    CUDA_TRY(cudaMemset(c->d_ws2, 0, sizeof(unsigned long long) * kWsSlots));
+                    CUDA_TRY(cudaMalloc(&c->d_ticket2, 64));
+                    CUDA_TRY(cudaMemset(c->d_ticket2, 0, 64));
+                    CUDA_TRY(cudaDeviceSynchronize());
+                    CUDA_TRY(cudaEventRecord(c->ev_fork, (cudaStream_t)stream));   // first use: after the contractions
+                    CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+                }
+                up_kparams R = P;
+                R.ws = c->d_ws2;
+                R.ticket = c->d_ticket2;
+                R.result = c->d_parts + (size_t)pl.prods.size() * LAs;
+                // one block per SM: it shares each SM with the contraction's CTA (launched first)
+                const int bps = pl.rest_kernel->blocks_per_sm;
+                pl.rest_kernel->blocks_per_sm = 1;
+                const up_status ls = launch(c, pl.rest_kernel, R, R.n, c->side);
+                pl.rest_kernel->blocks_per_sm = bps;
+                if (ls) return ls;
+                CUDA_TRY(cudaEventRecord(c->ev_join, c->side));
+            }
+            if (pl.rest_kernel && !overlap) {
                 P.result = c->d_parts + (size_t)ti++ * LAs;
                 if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream)) return s;
             }
+            if (overlap) CUDA_TRY(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_join, 0));
             CUDA_TRY(upk_launch_combine(c->d_parts, T, LAs, d_partial, (cudaStream_t)stream));
             c->launches++;
             return UP_OK;
