@@ -1148,12 +1148,12 @@ std::unique_ptr<Node> clone_node(const Node *n) {
 }  // namespace
 
 // SUM(root) = sum of SUM(+-ci*cj) over the top-level column-product terms at
-// the output scale (row contraction kernels) + SUM(rest) with the rest cast to
-// the output scale (fused per-thread kernel).  Exact: SUM is linear and every
+// the output scale (row contraction kernels) + 10^rest_scale * SUM(rest), the
+// rest summed at its own scale (fused per-thread kernel).  Exact: SUM is linear and every
 // term is an exact part of the row value.  Products below another scale, or
 // too small to be compute-bound, stay in the rest.
 bool split_sum_terms(const Node *root, const std::vector<ColType> &cols, int min_products,
-                     std::vector<SplitTerm> &prods, std::unique_ptr<Node> &rest) {
+                     std::vector<SplitTerm> &prods, std::unique_ptr<Node> &rest, int &rest_scale) {
     const Node *body = root->op == Op::Cast ? root->l.get() : root;
     const int s_out = root->s;
     std::vector<std::pair<int, const Node *>> terms;
@@ -1185,16 +1185,9 @@ bool split_sum_terms(const Node *root, const std::vector<ColType> &cols, int min
         std::string err;
         type_tree(acc.get(), cols, err);
         if (!err.empty() || acc->s > s_out) return false;
-        if (acc->s < s_out) {
-            auto cst = std::make_unique<Node>();
-            cst->op = Op::Cast;
-            cst->p = acc->p + (s_out - acc->s);
-            cst->s = s_out;
-            cst->L = limbs_for_precision(cst->p);
-            cst->l = std::move(acc);
-            acc = std::move(cst);
-            type_tree(acc.get(), cols, err);
-        }
+        // the rest is summed at its own scale; its partial is multiplied by
+        // 10^rest_scale in the combine (SUM is linear: no per-row alignment)
+        rest_scale = s_out - acc->s;
         rest = std::move(acc);
     }
     return true;

@@ -36,7 +36,7 @@ struct SplitTerm {
 std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int col_b, GenInfo &info);
 std::string gen_contract_kernel28(int La, int Lb, int LA, int sign, int col_a, int col_b, GenInfo &info);
 bool split_sum_terms(const Node *root, const std::vector<ColType> &cols, int min_products,
-                     std::vector<SplitTerm> &prods, std::unique_ptr<Node> &rest);
+                     std::vector<SplitTerm> &prods, std::unique_ptr<Node> &rest, int &rest_scale);
 // wide SUM regime (warp per row); "" if the expression does not fit it
 std::string gen_wide_sum_kernel(const Node *root, const std::vector<ColType> &cols, int LA, GenInfo &info);
 

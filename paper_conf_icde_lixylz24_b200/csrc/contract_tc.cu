@@ -36,11 +36,11 @@ namespace {
 typedef uint32_t u32;
 typedef unsigned long long u64;
 
-constexpr int THREADS = 256;
-constexpr int NRAW = 3;                  // raw (bulk-copied) stages in flight
+constexpr int THREADS = 512;            // transform warps (16); + 1 control warp
+constexpr int NRAW_MAX = 4;              // raw (TMA-filled) stages in flight, at most
 constexpr int MAX_SLOTS = 1024;
 constexpr int MAX_ROLE_LIMBS = 256;
-constexpr int ABOX = 32;                 // c_a limbs per M tile (128 digits)
+constexpr int ABOX_MAX = 32;             // c_a limbs per M tile (128 digits)
 
 struct TcArgs {
     const u32 *A, *B;
@@ -51,7 +51,8 @@ struct TcArgs {
     u32 *ticket;
     u32 *result;      // LA limbs
     int LA, nsl, sign;
-    int bbox;         // c_b limbs per N group box (<= 128)
+    int abox, bbox;   // c_a limbs per M-tile box (<= 32), c_b limbs per N-group box (<= 129)
+    int nst;          // raw stages (2..NRAW_MAX), as many as shared memory holds
 };
 
 __device__ __forceinline__ u32 smem_u32(const void *p) { return (u32)__cvta_generic_to_shared(p); }
@@ -104,11 +105,12 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
     constexpr int DRAIN_CHUNKS = 32768 / KC; // s32 accumulators drained every 32768 rows
     extern __shared__ __align__(1024) unsigned char smem[];
     __shared__ u32 s_taddr;
-    __shared__ __align__(8) u64 s_full[NRAW], s_empty[NRAW], s_cfull[2], s_mdone[2], s_drained;
+    __shared__ __align__(8) u64 s_full[NRAW_MAX], s_empty[NRAW_MAX], s_cfull[2], s_mdone[2], s_drained;
     __shared__ u32 s_last;
 
-    // warps 0-7 transform raw limb rows into the MMA layout (warps 0-3 also
-    // drain TMEM lanes 0-127); warp 8 issues the bulk copies and the MMAs
+    // warps 0..THREADS/32-1 transform raw limb rows into the MMA layout (warps
+    // 0-3 also drain TMEM lanes 0-127); the last warp issues the TMA copies and the MMAs
+    const int NRAW = P.nst;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int role = blockIdx.x % P.n_roles, rblock = blockIdx.x / P.n_roles;
     const int mt = role % P.n_mtiles, grp = role / P.n_mtiles;
@@ -130,9 +132,9 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
     ob.dbase = y0; ob.L = P.Lb; ob.lo = y0 / 4; ob.nl = max(0, min(P.Lb, (y0 + W) / 4) - ob.lo);
     ob.extra_top = (4 * P.Lb >= y0 && 4 * P.Lb < y0 + W) && ob.nl == 0;
     ob.ndig = ny;
-    ob.raw_off = ABOX;
+    ob.raw_off = P.abox;
     const int box_a = oa.extra_top ? P.La - 1 : oa.lo, box_b = ob.extra_top ? P.Lb - 1 : ob.lo;
-    const int nraw_limbs = ABOX + P.bbox;
+    const int nraw_limbs = P.abox + P.bbox;
 
     // shared: [NRAW raw stages: limb x KC words][2 canonical stages: A 128 x KC | B W x KC][digit sums]
     const int raw_bytes = nraw_limbs * KC * 4;
@@ -153,10 +155,10 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
     if (tid == 0) {
         for (int i = 0; i < NRAW; ++i) {
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&s_full[i])));
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;" :: "r"(smem_u32(&s_empty[i])));
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(&s_empty[i])), "r"(THREADS / 32));
         }
         for (int i = 0; i < 2; ++i) {
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;" :: "r"(smem_u32(&s_cfull[i])));
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(&s_cfull[i])), "r"(THREADS / 32));
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&s_mdone[i])));
         }
         asm volatile("mbarrier.init.shared::cta.b64 [%0], 4;" :: "r"(smem_u32(&s_drained)));
@@ -170,14 +172,13 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
     const long long n = P.n;
     const long long nchunks = (n + KC - 1) / KC;
     const long long my_chunks = rblock < nchunks ? (nchunks - 1 - rblock) / P.n_rblocks + 1 : 0;
-    auto is_drain = [&](long long t) { return ((t + 1) % DRAIN_CHUNKS) == 0 || t == my_chunks - 1; };
+    auto is_drain = [&](int t) { return ((t + 1) % DRAIN_CHUNKS) == 0 || t == (int)my_chunks - 1; };
 
-    if (warp == 8) {
+    if (warp == THREADS / 32) {
         // ---------------- control warp: bulk copies + MMA issue
-        auto issue = [&](long long t) {   // the role's limb rows of local chunk t -> raw stage t % NRAW (2 TMA boxes)
+        auto issue = [&](int t, int rs) {   // the role's limb rows of local chunk t -> raw stage rs = t % NRAW (2 TMA boxes)
             if (lane != 0) return;
-            const int rs = (int)(t % NRAW);
-            const int row0 = (int)((rblock + t * P.n_rblocks) * KC);
+            const int row0 = (int)((rblock + (long long)t * P.n_rblocks) * KC);
             const u32 mb = smem_u32(&s_full[rs]);
             const u32 tx = (u32)(nraw_limbs * KC * 4);
             asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(mb), "r"(tx) : "memory");
@@ -185,14 +186,15 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
             asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
                          :: "r"(dst), "l"(&tA), "r"(row0), "r"(box_a), "r"(mb) : "memory");
             asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
-                         :: "r"(dst + (u32)(ABOX * KC * 4)), "l"(&tB), "r"(row0), "r"(box_b), "r"(mb) : "memory");
+                         :: "r"(dst + (u32)(P.abox * KC * 4)), "l"(&tB), "r"(row0), "r"(box_b), "r"(mb) : "memory");
         };
-        for (long long t = 0; t < NRAW && t < my_chunks; ++t) issue(t);
+        for (int t = 0; t < NRAW && t < (int)my_chunks; ++t) issue(t, t);
         const u32 idesc0 = (2u << 4) | ((u32)(N0 >> 3) << 17) | ((128u >> 4) << 24);
         const u32 idesc1 = (2u << 4) | ((u32)(N1 >> 3) << 17) | ((128u >> 4) << 24);
-        int drains = 0;
-        for (long long t = 0; t < my_chunks; ++t) {
-            const int cs = (int)(t & 1), rs = (int)(t % NRAW);
+        int drains = 0, rs = 0;
+        u32 rph = 0;                                       // raw stage rs, its use parity
+        for (int t = 0; t < (int)my_chunks; ++t) {
+            const int cs = t & 1;
             if (lane == 0) {
                 mbar_wait(smem_u32(&s_cfull[cs]), (u32)((t >> 1) & 1));           // canonical stage written
                 const bool fresh = (t == 0) || is_drain(t - 1);
@@ -216,15 +218,16 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
                 }
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
                              :: "r"(smem_u32(&s_mdone[cs])));
-                if (t + NRAW < my_chunks) mbar_wait(smem_u32(&s_empty[rs]), (u32)((t / NRAW) & 1));   // raw stage read
+                if (t + NRAW < (int)my_chunks) mbar_wait(smem_u32(&s_empty[rs]), rph);   // raw stage read
             }
             __syncwarp();
-            if (t + NRAW < my_chunks) issue(t + NRAW);
+            if (t + NRAW < (int)my_chunks) issue(t + NRAW, rs);
+            if (++rs == NRAW) { rs = 0; rph ^= 1u; }
         }
     } else {
         // ---------------- transform warps: per-thread task list fixed for the whole run
-        constexpr int MAXT = 16;
-        const int sub = tid & 7, quarter = tid >> 3;      // 32 quarters, 8 lanes (digits) each
+        constexpr int MAXT = 16 * 256 / THREADS;
+        const int sub = tid & 7, quarter = tid >> 3;      // THREADS/8 quarters, 8 lanes (digits) each
         const int ga = (oa.ndig + 7) / 8, gb = (ob.ndig + 7) / 8;
         const int tasks = (ga + gb) * NRG;
         u32 t_src[MAXT], t_dst[MAXT];                      // raw word offset; canonical byte offset | b << 20 | rg << 24
@@ -232,7 +235,7 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
 #pragma unroll
         for (int k = 0; k < MAXT; ++k) {
             t_src[k] = 0; t_dst[k] = 0xFFFFFFFFu;
-            const int task = quarter + 32 * k;
+            const int task = quarter + (THREADS / 8) * k;
             if (task >= tasks) continue;
             nt = k + 1;
             const int g = task / NRG, rg = task % NRG;
@@ -250,9 +253,11 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
             t_dst[k] = (u32)((isA ? 0 : a_bytes) + (dl >> 3) * SBO + rg * 128 + (dl & 7) * 16) | ((u32)sgn << 20);
         }
         const u32 sel = (u32)(sub & 3) | ((u32)(4 + (sub & 3)) << 4);   // this lane's byte of every word
-        for (long long t = 0; t < my_chunks; ++t) {
-            const int rs = (int)(t % NRAW), cs = (int)(t & 1);
-            mbar_wait(smem_u32(&s_full[rs]), (u32)((t / NRAW) & 1));               // raw rows landed
+        int rs = 0;
+        u32 rph = 0;
+        for (int t = 0; t < (int)my_chunks; ++t, rs = (rs + 1 == NRAW) ? 0 : rs + 1, rph ^= (rs == 0) ? 1u : 0u) {
+            const int cs = t & 1;
+            mbar_wait(smem_u32(&s_full[rs]), rph);                                  // raw rows landed
             if (t >= 2) mbar_wait(smem_u32(&s_mdone[cs]), (u32)(((t - 2) >> 1) & 1));  // canonical stage free
             const u32 *raw = reinterpret_cast<const u32 *>(raw0 + rs * raw_bytes);
             unsigned char *canon = canon0 + cs * st_bytes;
@@ -397,12 +402,16 @@ cudaError_t make_tmap(CUtensorMap *m, const u32 *data, long long n, int L, long 
 template <int KC>
 cudaError_t launch_kc(TcArgs P, int W, int nraw_limbs, int num_sms, cudaStream_t st) {
     CUtensorMap tA, tB;
-    cudaError_t e0 = make_tmap(&tA, P.A, P.n, P.La, P.lda, KC, ABOX);
+    cudaError_t e0 = make_tmap(&tA, P.A, P.n, P.La, P.lda, KC, P.abox);
     if (e0 != cudaSuccess) return e0;
     e0 = make_tmap(&tB, P.B, P.n, P.Lb, P.ldb, KC, P.bbox);
     if (e0 != cudaSuccess) return e0;
     const size_t sums = sizeof(u64) * (size_t)(2 * (128 + W));
-    size_t smem = (size_t)NRAW * nraw_limbs * KC * 4 + 2 * (size_t)(128 + W) * KC + sums;
+    const size_t fixed = 2 * (size_t)(128 + W) * KC + sums;
+    P.nst = NRAW_MAX;
+    while (P.nst > 2 && (size_t)P.nst * nraw_limbs * KC * 4 + fixed > 225 * 1024) --P.nst;
+    size_t smem = (size_t)P.nst * nraw_limbs * KC * 4 + fixed;
+    if (smem > 225 * 1024) return cudaErrorInvalidValue;
     if (smem < sizeof(u64) * 2 * (size_t)P.nsl) smem = sizeof(u64) * 2 * (size_t)P.nsl;
     cudaError_t e = cudaFuncSetAttribute(k_contract_tc<KC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -446,11 +455,12 @@ cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, con
     const int W = ((MB < 512 ? MB : 512) + 15) & ~15;
     P.bbox = (W / 4 < Lb ? W / 4 : Lb) + 1;               // group limbs (+1: a sign-only tile starts one limb early)
     if (P.bbox > 128 + 1) P.bbox = 129;
-    const int nraw = ABOX + P.bbox;
+    P.abox = La < ABOX_MAX ? La : ABOX_MAX;
+    const int nraw = P.abox + P.bbox;
     if (nraw > MAX_ROLE_LIMBS) return cudaErrorInvalidValue;
     // stage depth: 128 rows when the role's raw + canonical stages fit, else 64
-    const size_t need128 = (size_t)NRAW * nraw * 128 * 4 + 2 * (size_t)(128 + W) * 128;
-    const int max_tasks = (16 + (W + 7) / 8) * (128 / 16);   // transform tasks per 128-row stage (<= 32 x MAXT)
+    const size_t need128 = (size_t)3 * nraw * 128 * 4 + 2 * (size_t)(128 + W) * 128;   // >= 3 raw stages at 128 rows
+    const int max_tasks = (16 + (W + 7) / 8) * (128 / 16);   // transform tasks per 128-row stage (<= 512)
     if (need128 + 16 * 1024 <= 220 * 1024 && max_tasks <= 512) return launch_kc<128>(P, W, nraw, num_sms, st);
     return launch_kc<64>(P, W, nraw, num_sms, st);
 }

@@ -78,6 +78,39 @@ __global__ void __launch_bounds__(1024) k_combine(const u32 *__restrict__ parts,
     }
 }
 
+// Split-SUM combine: out = sum of the partials, partial `scaled` multiplied by
+// the unsigned constant scale[0..nsc) first (two's complement mod 2^(32 la):
+// exact).  Column j: 64-bit sums of the low and high halves of its products,
+// then one carry pass.
+__global__ void __launch_bounds__(1024) k_combine_scaled(const u32 *__restrict__ parts, int nparts, int la, int scaled,
+                                                         const u32 *__restrict__ scale, int nsc, u32 *__restrict__ out) {
+    extern __shared__ u64 col[];
+    u64 *hi = col + la;
+    const u32 *sp = parts + (long long)scaled * la;
+    for (int j = threadIdx.x; j < la; j += blockDim.x) {
+        u64 lo = 0, h = 0;
+        for (int r = 0; r < nparts; ++r)
+            if (r != scaled) lo += parts[(long long)r * la + j];
+        for (int m = 0; m < nsc && m <= j; ++m) {
+            const u64 pr = (u64)sp[j - m] * scale[m];
+            lo += (u32)pr;
+            h += pr >> 32;
+        }
+        col[j] = lo;
+        hi[j] = h;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        u64 carry = 0;
+        for (int j = 0; j < la; ++j) {
+            // value at limb j: lo[j] + hi[j] 2^32 (+ carry from below)
+            const u64 t = (col[j] & 0xffffffffull) + carry;
+            out[j] = (u32)t;
+            carry = (t >> 32) + (col[j] >> 32) + hi[j];
+        }
+    }
+}
+
 // Compact byte-aligned rows (the paper's cDecimal, P:L843-873 / Fig. 4):
 // Lb bytes per row, little-endian magnitude, the sign in the top bit of the
 // last byte.  A block stages its 256 contiguous records with 32-bit loads
@@ -214,6 +247,17 @@ cudaError_t upk_launch_combine(const uint32_t *partials, int nranks, int la, uin
         if (e != cudaSuccess) return e;
     }
     k_combine<<<1, 1024, smem, st>>>(partials, nranks, la, out);
+    return cudaGetLastError();
+}
+
+cudaError_t upk_launch_combine_scaled(const uint32_t *partials, int nparts, int la, uint32_t *out, int scaled,
+                                      const uint32_t *scale, int nsc, cudaStream_t st) {
+    const size_t smem = 2 * sizeof(u64) * (size_t)la;
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(k_combine_scaled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    k_combine_scaled<<<1, 1024, smem, st>>>(partials, nparts, la, scaled, scale, nsc, out);
     return cudaGetLastError();
 }
 

@@ -37,6 +37,8 @@ cudaError_t upk_launch_from_bin(const uint32_t *mag, int W, const uint8_t *neg, 
 cudaError_t upk_launch_to_bin(const uint32_t *planes, int L, long long ld, long long n, uint32_t *mag, uint8_t *neg,
                               cudaStream_t st);
 cudaError_t upk_launch_combine(const uint32_t *partials, int nranks, int la, uint32_t *out, cudaStream_t st);
+cudaError_t upk_launch_combine_scaled(const uint32_t *partials, int nparts, int la, uint32_t *out, int scaled,
+                                      const uint32_t *scale, int nsc, cudaStream_t st);
 int upk_contract_tc_slots(int La, int Lb);
 cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, const uint32_t *B, long long ldb, int Lb,
                                    long long n, int sign, unsigned long long *ws, uint32_t *ticket, uint32_t *result,
@@ -139,6 +141,7 @@ struct SplitPlan {
     std::vector<uph::SplitTerm> prods;
     std::vector<JitKernel *> cc_kernels;   // per product: CUDA-core kernel, nullptr = tensor cores
     JitKernel *rest_kernel = nullptr;
+    int rest_scale = 0;                    // rest partial x 10^rest_scale in the combine
 };
 
 struct up_ctx {
@@ -757,7 +760,7 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(ts.root.get(), ts.types);
             const Node *base = opt_root ? opt_root.get() : ts.root.get();
             std::unique_ptr<Node> rest;
-            pl.split = pl.LAs <= 512 && split_sum_terms(base, ts.types, kContractMinProducts, pl.prods, rest);
+            pl.split = pl.LAs <= 512 && split_sum_terms(base, ts.types, kContractMinProducts, pl.prods, rest, pl.rest_scale);
             if (pl.split) {
                 const int LAs = pl.LAs;
                 for (const SplitTerm &st : pl.prods) {
@@ -859,7 +862,14 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
                 if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream)) return s;
             }
             if (overlap) CUDA_TRY(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_join, 0));
-            CUDA_TRY(upk_launch_combine(c->d_parts, T, LAs, d_partial, (cudaStream_t)stream));
+            if (pl.rest_kernel && pl.rest_scale > 0) {
+                const uint32_t *d_sc = nullptr;
+                if (up_status s = pow10_device(c, pl.rest_scale, &d_sc)) return s;
+                CUDA_TRY(upk_launch_combine_scaled(c->d_parts, T, LAs, d_partial, T - 1, d_sc,
+                                                   limbs_for_precision(pl.rest_scale), (cudaStream_t)stream));
+            } else {
+                CUDA_TRY(upk_launch_combine(c->d_parts, T, LAs, d_partial, (cudaStream_t)stream));
+            }
             c->launches++;
             return UP_OK;
         }
