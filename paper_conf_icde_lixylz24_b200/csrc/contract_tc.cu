@@ -171,14 +171,17 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
 
     const long long n = P.n;
     const long long nchunks = (n + KC - 1) / KC;
-    const long long my_chunks = rblock < nchunks ? (nchunks - 1 - rblock) / P.n_rblocks + 1 : 0;
+    // a contiguous range of chunks per row block: consecutive stages read
+    // consecutive segments of every limb plane
+    const long long c_begin = nchunks * rblock / P.n_rblocks, c_end = nchunks * (rblock + 1) / P.n_rblocks;
+    const long long my_chunks = c_end - c_begin;
     auto is_drain = [&](int t) { return ((t + 1) % DRAIN_CHUNKS) == 0 || t == (int)my_chunks - 1; };
 
     if (warp == THREADS / 32) {
         // ---------------- control warp: bulk copies + MMA issue
         auto issue = [&](int t, int rs) {   // the role's limb rows of local chunk t -> raw stage rs = t % NRAW (2 TMA boxes)
             if (lane != 0) return;
-            const int row0 = (int)((rblock + (long long)t * P.n_rblocks) * KC);
+            const int row0 = (int)((c_begin + t) * KC);
             const u32 mb = smem_u32(&s_full[rs]);
             const u32 tx = (u32)(nraw_limbs * KC * 4);
             asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(mb), "r"(tx) : "memory");
