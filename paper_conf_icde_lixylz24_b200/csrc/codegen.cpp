@@ -44,14 +44,16 @@ int mag_limbs_of_pow10(int k) {   // limbs of the magnitude 10^k - 1 (at least 1
 }
 
 // Window of the top-limb division decision (div_top_decide in up_dev.cuh):
-// T divisor limbs, T = max(limbs(C), limbs(q)) + 2 so that an undecided row
-// has probability ~2^-64 for a full-length divisor; used when the divisor is
-// wider than the window and the dividend reaches into it.  Returns T, or 0.
+// T divisor limbs, T = max(limbs(C), limbs(q)) + 1 (UP_DIVTOP_T2: + 2), so an
+// undecided row has probability ~(q0 + C)/v_h, below 2^-30 for a divisor whose
+// top limb is not tiny (cfg3: ~2^-33); undecided rows run the full division,
+// so the window only trades speed.  Used when the divisor is wider than the
+// window and the dividend reaches into it.  Returns T, or 0.
 int div_top_window(const Node *n) {
     if (n->op != Op::Div || getenv("UP_NO_DIVTOP")) return 0;
     const int La = n->l->L, Lb = n->r->L;
     const int NC = (int)HBig::pow10(n->r->s + 4).w.size();
-    const int T = std::max(NC, n->L) + 2;
+    const int T = std::max(NC, n->L) + (getenv("UP_DIVTOP_T2") ? 2 : 1);
     const int E = Lb - T;
     return (E > 0 && La > E) ? T : 0;
 }
