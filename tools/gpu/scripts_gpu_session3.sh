@@ -5,7 +5,7 @@ O=gpurun_out/s3; mkdir -p $O
 nvidia-smi --query-gpu=name,driver_version,clocks.sm,clocks.max.sm,power.limit --format=csv > $O/gpu.txt 2>&1
 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log
 timeout 1800 python -m pytest tests -q -p no:cacheprovider -m gpu > $O/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $O/pytest_gpu.log
-O=$O/bench PARTS=1 ./scripts_gpu_bench_all.sh
+O=$O/bench PARTS=1 ./tools/gpu/scripts_gpu_bench_all.sh
 timeout 600 python bench.py --impl reference > $O/bench_reference_cfg2.log 2>&1
 for c in 2 3 4 5; do
   R=""; [ $c = 4 ] && R="--rows 1000000"; [ $c = 5 ] && R="--rows 100000"
