@@ -737,7 +737,8 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     // With the tensor-core contraction (contract_tc.cu, default; UP_NO_TC for
     // the CUDA-core one) every top-level column product of >= kContractMinProducts
     // limb products is split off.
-    const bool use_tc = getenv("UP_NO_TC") == nullptr;
+    // (TMA row coordinates are 32-bit signed: more rows per call take the CUDA-core contraction)
+    const bool use_tc = getenv("UP_NO_TC") == nullptr && cols[0].n < (1ll << 31);
     bool try_split = getenv("UP_SPLIT") != nullptr;
     if (!try_split && !getenv("UP_NO_SPLIT")) {
         const long thr = use_tc ? kContractMinProducts : kSplitAutoProducts;
