@@ -57,10 +57,11 @@ struct TcArgs {
 
 __device__ __forceinline__ u32 smem_u32(const void *p) { return (u32)__cvta_generic_to_shared(p); }
 
-// K-major, no swizzle: LBO = 128 B (next 16-byte K chunk), SBO = next 8-row group
-template <int SBO>
-__device__ __forceinline__ u64 umma_desc(u32 saddr) {
-    return (u64)((saddr >> 4) & 0x3FFFu) | ((u64)(128 >> 4) << 16) | ((u64)(SBO >> 4) << 32) | (1ull << 46);
+// MN-major, no swizzle: a core matrix is 16 digit bytes (MN) x 8 rows (K),
+// 128 B; SBO = 128 B (next 16-digit chunk), LBO = next 8-row group
+// (chunks x 128 B).  Verified against a host GEMM by tools/tc_probe.cu.
+__device__ __forceinline__ u64 umma_desc_mn(u32 saddr, u32 lbo) {
+    return (u64)((saddr >> 4) & 0x3FFFu) | ((u64)((lbo >> 4) & 0x3FFFu) << 16) | ((u64)(128 >> 4) << 32) | (1ull << 46);
 }
 
 // bounded wait: a lost completion traps (launch error) instead of hanging.
@@ -81,13 +82,6 @@ __device__ __forceinline__ void mbar_wait(u32 mb, u32 parity) {
     }
 }
 
-// byte b of four words -> one word (b < 4), or their sign bits (b == 4)
-__device__ __forceinline__ u32 pick4(u32 x0, u32 x1, u32 x2, u32 x3, int b) {
-    if (b == 4) return (x0 >> 31) | ((x1 >> 31) << 8) | ((x2 >> 31) << 16) | ((x3 >> 31) << 24);
-    const u32 sel = (u32)b | ((u32)(4 + b) << 4);
-    return __byte_perm(__byte_perm(x0, x1, sel), __byte_perm(x2, x3, sel), 0x5410);
-}
-
 // A role's operand tile: digits [dbase, dbase + extent) of one column; its raw
 // stage holds the limbs lo .. lo + nl - 1 (+ the top limb when only the sign
 // digit falls into the tile)
@@ -100,8 +94,6 @@ struct Opnd {
 template <int KC>
 __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P, const __grid_constant__ CUtensorMap tA,
                                                                   const __grid_constant__ CUtensorMap tB) {
-    constexpr int NRG = KC / 16;             // 16-row groups per stage
-    constexpr int SBO = NRG * 128;           // bytes between 8-digit core-matrix groups
     constexpr int DRAIN_CHUNKS = 32768 / KC; // s32 accumulators drained every 32768 rows
     extern __shared__ __align__(1024) unsigned char smem[];
     __shared__ u32 s_taddr;
@@ -139,6 +131,7 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
     // shared: [NRAW raw stages: limb x KC words][2 canonical stages: A 128 x KC | B W x KC][digit sums]
     const int raw_bytes = nraw_limbs * KC * 4;
     const int a_bytes = 128 * KC, b_bytes = W * KC, st_bytes = a_bytes + b_bytes;
+    const u32 LBO_A = (128 / 16) * 128, LBO_B = (u32)(W / 16) * 128;   // bytes per 8-row group of a tile
     unsigned char *raw0 = smem;
     unsigned char *canon0 = smem + NRAW * raw_bytes;
     const int ND = 128 + W;
@@ -192,8 +185,9 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
                          :: "r"(dst + (u32)(P.abox * KC * 4)), "l"(&tB), "r"(row0), "r"(box_b), "r"(mb) : "memory");
         };
         for (int t = 0; t < NRAW && t < (int)my_chunks; ++t) issue(t, t);
-        const u32 idesc0 = (2u << 4) | ((u32)(N0 >> 3) << 17) | ((128u >> 4) << 24);
-        const u32 idesc1 = (2u << 4) | ((u32)(N1 >> 3) << 17) | ((128u >> 4) << 24);
+        // s32 accumulate, u8 x u8, A and B MN-major (bits 15, 16)
+        const u32 idesc0 = (2u << 4) | (1u << 15) | (1u << 16) | ((u32)(N0 >> 3) << 17) | ((128u >> 4) << 24);
+        const u32 idesc1 = (2u << 4) | (1u << 15) | (1u << 16) | ((u32)(N1 >> 3) << 17) | ((128u >> 4) << 24);
         int drains = 0, rs = 0;
         u32 rph = 0;                                       // raw stage rs, its use parity
         for (int t = 0; t < (int)my_chunks; ++t) {
@@ -207,13 +201,13 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
 #pragma unroll
                 for (int kk = 0; kk < KC / 32; ++kk) {
                     const u32 acc = (!fresh || kk > 0) ? 1u : 0u;
-                    const u64 da = umma_desc<SBO>(a_addr + kk * 256);
-                    const u64 db0 = umma_desc<SBO>(b_addr + kk * 256);
+                    const u64 da = umma_desc_mn(a_addr + kk * 4 * LBO_A, LBO_A);
+                    const u64 db0 = umma_desc_mn(b_addr + kk * 4 * LBO_B, LBO_B);
                     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                                  "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}\n"
                                  :: "r"(taddr), "l"(da), "l"(db0), "r"(idesc0), "r"(acc));
                     if (N1 > 0) {
-                        const u64 db1 = umma_desc<SBO>(b_addr + (N0 / 8) * SBO + kk * 256);
+                        const u64 db1 = umma_desc_mn(b_addr + (N0 / 16) * 128 + kk * 4 * LBO_B, LBO_B);
                         asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                                      "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}\n"
                                      :: "r"(taddr + (u32)N0), "l"(da), "l"(db1), "r"(idesc1), "r"(acc));
@@ -228,34 +222,49 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
             if (++rs == NRAW) { rs = 0; rph ^= 1u; }
         }
     } else {
-        // ---------------- transform warps: per-thread task list fixed for the whole run
-        constexpr int MAXT = 16 * 256 / THREADS;
-        const int sub = tid & 7, quarter = tid >> 3;      // THREADS/8 quarters, 8 lanes (digits) each
-        const int ga = (oa.ndig + 7) / 8, gb = (ob.ndig + 7) / 8;
-        const int tasks = (ga + gb) * NRG;
-        u32 t_src[MAXT], t_dst[MAXT];                      // raw word offset; canonical byte offset | b << 20 | rg << 24
+        // ---------------- transform warps: word transpose into the MN-major layout.
+        // Task = (16-digit chunk c of a tile, row r): the chunk's bytes in row r
+        // are the little-endian words of limbs 4c..4c+3 -> 4 LDS.32 (consecutive
+        // rows across lanes) and one STS.128 (lanes 16 B apart: conflict-free).
+        // The word at the sign digit's position is the row's sign bit; words of
+        // limbs beyond the column stay zero.  Task list fixed for the whole run.
+        constexpr int MAXT = 10;                                        // (8 + 32) chunks x 128 rows / 512 threads
+        const int ca_used = min(8, (oa.ndig + 15) / 16), cb_used = (ob.ndig + 15) / 16;
+        const int tasks = (ca_used + cb_used) * KC;
+        u32 t_src[MAXT], t_dst[MAXT], t_mode[MAXT];   // raw word offset of the first word; canonical byte offset; word kinds
         int nt = 0;
 #pragma unroll
         for (int k = 0; k < MAXT; ++k) {
-            t_src[k] = 0; t_dst[k] = 0xFFFFFFFFu;
-            const int task = quarter + (THREADS / 8) * k;
+            t_src[k] = 0; t_dst[k] = 0; t_mode[k] = 0;
+            const int task = tid + THREADS * k;
             if (task >= tasks) continue;
             nt = k + 1;
-            const int g = task / NRG, rg = task % NRG;
-            const bool isA = g < ga;
+            const int cidx = task / KC, r = task % KC;
+            const bool isA = cidx < ca_used;
             const Opnd &o = isA ? oa : ob;
-            const int dl = 8 * (isA ? g : g - ga) + sub;
-            if (dl >= o.ndig) continue;
-            const int d = o.dbase + dl;
+            const int c = isA ? cidx : cidx - ca_used;
             const int blo = isA ? box_a : box_b;
-            int sgn, slot;
-            if (d < 4 * o.L) { sgn = 0; slot = d / 4 - blo; }         // byte d & 3 == sub & 3 (tiles start at multiples of 4)
-            else if (d == 4 * o.L) { sgn = 1; slot = o.L - 1 - blo; }
-            else continue;
-            t_src[k] = (u32)((o.raw_off + slot) * KC + 16 * rg);
-            t_dst[k] = (u32)((isA ? 0 : a_bytes) + (dl >> 3) * SBO + rg * 128 + (dl & 7) * 16) | ((u32)sgn << 20);
+            const int nbox = isA ? P.abox : P.bbox;
+            // word q of the chunk = limb (dbase/4 + 4c + q); kinds: 0 normal, 1 sign, 2 zero
+            u32 mode = 0;
+            int first_slot = -1;
+            for (int q = 0; q < 4; ++q) {
+                const int lj = o.dbase / 4 + 4 * c + q;        // global limb index of this word
+                u32 kind;
+                if (lj < o.L) kind = 0;
+                else if (lj == o.L) kind = 1;
+                else kind = 2;
+                if (kind == 0 && first_slot < 0) first_slot = lj - blo;
+                mode |= kind << (2 * q);
+            }
+            // sign word reads the top limb's slot
+            const int sign_slot = o.L - 1 - blo;
+            if (first_slot < 0) first_slot = sign_slot;          // chunk holding only the sign digit
+            (void)nbox;
+            t_src[k] = (u32)((o.raw_off + first_slot) * KC + r) | ((u32)(sign_slot - first_slot + 8) << 24);
+            t_dst[k] = (u32)((isA ? 0 : a_bytes) + (r >> 3) * (int)(isA ? LBO_A : LBO_B) + c * 128 + (r & 7) * 16);
+            t_mode[k] = mode;
         }
-        const u32 sel = (u32)(sub & 3) | ((u32)(4 + (sub & 3)) << 4);   // this lane's byte of every word
         int rs = 0;
         u32 rph = 0;
         for (int t = 0; t < (int)my_chunks; ++t, rs = (rs + 1 == NRAW) ? 0 : rs + 1, rph ^= (rs == 0) ? 1u : 0u) {
@@ -267,25 +276,22 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
 #pragma unroll
             for (int k = 0; k < MAXT; ++k) {
                 if (k >= nt) break;
-                const u32 td = t_dst[k];
-                if (td == 0xFFFFFFFFu) continue;
-                const uint4 *src = reinterpret_cast<const uint4 *>(raw + t_src[k]);
-                uint4 w[4];
-#pragma unroll
-                for (int q = 0; q < 4; ++q) w[q] = src[q];
+                const u32 src = t_src[k] & 0xFFFFFFu, mode = t_mode[k];
                 uint4 out;
-                if (!(td >> 20)) {
-                    out.x = __byte_perm(__byte_perm(w[0].x, w[0].y, sel), __byte_perm(w[0].z, w[0].w, sel), 0x5410);
-                    out.y = __byte_perm(__byte_perm(w[1].x, w[1].y, sel), __byte_perm(w[1].z, w[1].w, sel), 0x5410);
-                    out.z = __byte_perm(__byte_perm(w[2].x, w[2].y, sel), __byte_perm(w[2].z, w[2].w, sel), 0x5410);
-                    out.w = __byte_perm(__byte_perm(w[3].x, w[3].y, sel), __byte_perm(w[3].z, w[3].w, sel), 0x5410);
-                } else {                                   // sign digit: top bit of the top limb
-                    out.x = pick4(w[0].x, w[0].y, w[0].z, w[0].w, 4);
-                    out.y = pick4(w[1].x, w[1].y, w[1].z, w[1].w, 4);
-                    out.z = pick4(w[2].x, w[2].y, w[2].z, w[2].w, 4);
-                    out.w = pick4(w[3].x, w[3].y, w[3].z, w[3].w, 4);
+                if (mode == 0) {                                // the common case: 4 limbs of the column
+                    out.x = raw[src]; out.y = raw[src + KC]; out.z = raw[src + 2 * KC]; out.w = raw[src + 3 * KC];
+                } else {
+                    const int sdel = (int)(t_src[k] >> 24) - 8;
+                    const u32 sgn = raw[(int)src + sdel * KC] >> 31;
+                    u32 wq[4];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const u32 kind = (mode >> (2 * q)) & 3u;
+                        wq[q] = kind == 0 ? raw[src + q * KC] : kind == 1 ? sgn : 0u;
+                    }
+                    out = make_uint4(wq[0], wq[1], wq[2], wq[3]);
                 }
-                *reinterpret_cast<uint4 *>(canon + (td & 0xFFFFFu)) = out;
+                *reinterpret_cast<uint4 *>(canon + t_dst[k]) = out;
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             __syncwarp();
@@ -463,8 +469,8 @@ cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, con
     if (nraw > MAX_ROLE_LIMBS) return cudaErrorInvalidValue;
     // stage depth: 128 rows when the role's raw + canonical stages fit, else 64
     const size_t need128 = (size_t)3 * nraw * 128 * 4 + 2 * (size_t)(128 + W) * 128;   // >= 3 raw stages at 128 rows
-    const int max_tasks = (16 + (W + 7) / 8) * (128 / 16);   // transform tasks per 128-row stage (<= 512)
-    if (need128 + 16 * 1024 <= 220 * 1024 && max_tasks <= 512) return launch_kc<128>(P, W, nraw, num_sms, st);
+    const int max_tasks = (8 + W / 16) * 128;             // transform tasks per 128-row stage (<= 512 x MAXT)
+    if (need128 + 16 * 1024 <= 220 * 1024 && max_tasks <= 5120) return launch_kc<128>(P, W, nraw, num_sms, st);
     return launch_kc<64>(P, W, nraw, num_sms, st);
 }
 

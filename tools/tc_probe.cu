@@ -24,14 +24,27 @@ __global__ void probe(const uint8_t *A, const uint8_t *B, int N, int lbo_mode, u
     __shared__ u32 s_taddr;
     __shared__ __align__(8) u64 mbar;
     const int tid = threadIdx.x;
-    // SBO = 256 (an 8-row group holds 2 K chunks of 128 B), LBO = 128
-    for (int i = tid; i < 128 * 32; i += blockDim.x) {
-        const int r = i / 32, k = i % 32;
-        sa[(r >> 3) * 256 + (k >> 4) * 128 + (r & 7) * 16 + (k & 15)] = A[i];
-    }
-    for (int i = tid; i < N * 32; i += blockDim.x) {
-        const int r = i / 32, k = i % 32;
-        sb[(r >> 3) * 256 + (k >> 4) * 128 + (r & 7) * 16 + (k & 15)] = B[i];
+    if (lbo_mode < 2) {
+        // K-major: SBO = 256 (an 8-row group holds 2 K chunks of 128 B), LBO = 128
+        for (int i = tid; i < 128 * 32; i += blockDim.x) {
+            const int r = i / 32, k = i % 32;
+            sa[(r >> 3) * 256 + (k >> 4) * 128 + (r & 7) * 16 + (k & 15)] = A[i];
+        }
+        for (int i = tid; i < N * 32; i += blockDim.x) {
+            const int r = i / 32, k = i % 32;
+            sb[(r >> 3) * 256 + (k >> 4) * 128 + (r & 7) * 16 + (k & 15)] = B[i];
+        }
+    } else {
+        // MN-major: core matrix = 16 MN-contiguous bytes x 8 K rows (128 B);
+        // MN chunks 128 B apart, 8-row K groups (M/16)*128 B apart
+        for (int i = tid; i < 128 * 32; i += blockDim.x) {
+            const int m = i / 32, k = i % 32;
+            sa[(k >> 3) * (128 / 16) * 128 + (m >> 4) * 128 + (k & 7) * 16 + (m & 15)] = A[i];
+        }
+        for (int i = tid; i < N * 32; i += blockDim.x) {
+            const int m = i / 32, k = i % 32;
+            sb[(k >> 3) * (N / 16) * 128 + (m >> 4) * 128 + (k & 7) * 16 + (m & 15)] = B[i];
+        }
     }
     if (tid < 32) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 256;" :: "r"(smem_u32(&s_taddr)));
@@ -47,9 +60,18 @@ __global__ void probe(const uint8_t *A, const uint8_t *B, int N, int lbo_mode, u
     asm volatile("tcgen05.fence::after_thread_sync;");
     const u32 taddr = s_taddr;
     if (tid == 0) {
-        const u32 idesc = (2u << 4) | ((u32)(N >> 3) << 17) | ((128u >> 4) << 24);
-        const int lbo = lbo_mode ? 128 : 256, sbo = lbo_mode ? 256 : 128;   // mode 0: fields swapped
-        const u64 da = desc(smem_u32(sa), lbo, sbo), db = desc(smem_u32(sb), lbo, sbo);
+        u32 idesc = (2u << 4) | ((u32)(N >> 3) << 17) | ((128u >> 4) << 24);
+        u64 da, db;
+        if (lbo_mode < 2) {
+            const int lbo = lbo_mode ? 128 : 256, sbo = lbo_mode ? 256 : 128;   // mode 0: fields swapped
+            da = desc(smem_u32(sa), lbo, sbo); db = desc(smem_u32(sb), lbo, sbo);
+        } else {
+            idesc |= (1u << 15) | (1u << 16);                                   // A, B MN-major
+            // mode 2: LBO = K-group stride, SBO = MN-chunk stride; mode 3: swapped
+            const int ka = (128 / 16) * 128, kb = (N / 16) * 128;
+            if (lbo_mode == 2) { da = desc(smem_u32(sa), ka, 128); db = desc(smem_u32(sb), kb, 128); }
+            else { da = desc(smem_u32(sa), 128, ka); db = desc(smem_u32(sb), 128, kb); }
+        }
         asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                      "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}\n"
                      :: "r"(taddr), "l"(da), "l"(db), "r"(idesc), "r"(0u));
@@ -79,7 +101,7 @@ __global__ void probe(const uint8_t *A, const uint8_t *B, int N, int lbo_mode, u
 
 int main() {
     for (int N : {96, 256, 16}) {
-        for (int lbo_mode = 1; lbo_mode >= 0; --lbo_mode) {
+        for (int lbo_mode : {1, 2, 3}) {
             std::vector<uint8_t> A(128 * 32), B(N * 32);
             srand(N + lbo_mode);
             for (auto &x : A) x = rand() & 255;
@@ -103,7 +125,7 @@ int main() {
                     for (int k = 0; k < 32; ++k) ref += (u32)A[m * 32 + k] * B[n * 32 + k];
                     if (ref != D[m * N + n]) { if (first < 0) first = m * N + n; ++bad; }
                 }
-            printf("N=%d lbo=%d err=%s status=%d mismatches=%ld first=%ld", N, lbo_mode ? 128 : 256,
+            printf("N=%d mode=%d err=%s status=%d mismatches=%ld first=%ld", N, lbo_mode,
                    cudaGetErrorString(e), st, bad, first);
             if (first >= 0) {
                 const int m = first / N, n = first % N;
