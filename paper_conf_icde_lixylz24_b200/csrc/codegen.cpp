@@ -277,7 +277,14 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
         if (E.is_lazy(x)) return 0;
         return std::max(x->L, std::max(live(x->l.get()), live(x->r.get())));
     };
-    k << "extern \"C\" __global__ void " << launch_bounds(256, (R == 1 && live(root) <= 64) ? 2 : 0) << " upk(const up_kparams P) {\n";
+    // occupancy: a kernel whose wide columns are all read lazily by top-limb
+    // divisions keeps a narrow state per row -> 4 blocks/SM (64 registers; the
+    // rare full-division fallback spills).  Measured on cfg3's rest kernel:
+    // 2 -> 4 blocks/SM 1.227 -> 1.145 ms per step (profiles/r01_minblocks/).
+    bool any_lazy = false;
+    for (size_t c = 0; c < cols.size(); ++c) any_lazy = any_lazy || E.lazy[c];
+    const int min_blocks = (R == 1 && any_lazy && live(root) <= 16) ? 4 : (R == 1 && live(root) <= 64) ? 2 : 0;
+    k << "extern \"C\" __global__ void " << launch_bounds(256, min_blocks) << " upk(const up_kparams P) {\n";
     k << "    constexpr int R = " << R << ";\n";
     k << "    u32 fl = 0;\n";
     if (opt.sum) {
