@@ -228,7 +228,7 @@ __global__ void __launch_bounds__(THREADS + 32, 1) k_contract_tc(const TcArgs P,
         // rows across lanes) and one STS.128 (lanes 16 B apart: conflict-free).
         // The word at the sign digit's position is the row's sign bit; words of
         // limbs beyond the column stay zero.  Task list fixed for the whole run.
-        constexpr int MAXT = 10;                                        // (8 + 32) chunks x 128 rows / 512 threads
+        constexpr int MAXT = KC == 256 ? 16 : 10;                       // (8 + 32) chunks x 128 rows / 512 threads
         const int ca_used = min(8, (oa.ndig + 15) / 16), cb_used = (ob.ndig + 15) / 16;
         const int tasks = (ca_used + cb_used) * KC;
         u32 t_src[MAXT], t_dst[MAXT], t_mode[MAXT];   // raw word offset of the first word; canonical byte offset; word kinds
@@ -467,9 +467,17 @@ cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, con
     P.abox = La < ABOX_MAX ? La : ABOX_MAX;
     const int nraw = P.abox + P.bbox;
     if (nraw > MAX_ROLE_LIMBS) return cudaErrorInvalidValue;
-    // stage depth: 128 rows when the role's raw + canonical stages fit, else 64
+    // stage depth (measured on B200, profiles/r01_kc/): 256 rows when 2 raw + 2
+    // canonical stages fit (cfg3 p = 200: 1.098e10 -> 1.128e10 rows/s), else
+    // 128 rows with >= 3 raw stages, else 64
+    const size_t need256 = (size_t)2 * nraw * 256 * 4 + 2 * (size_t)(128 + W) * 256;
     const size_t need128 = (size_t)3 * nraw * 128 * 4 + 2 * (size_t)(128 + W) * 128;   // >= 3 raw stages at 128 rows
     const int max_tasks = (8 + W / 16) * 128;             // transform tasks per 128-row stage (<= 512 x MAXT)
+    if (const char *kc = getenv("UP_TC_KC")) {              // experiments: force the stage depth
+        if (atoi(kc) == 256) return launch_kc<256>(P, W, nraw, num_sms, st);
+        if (atoi(kc) == 64) return launch_kc<64>(P, W, nraw, num_sms, st);
+    }
+    if (need256 + 16 * 1024 <= 220 * 1024 && max_tasks * 2 <= 512 * 16) return launch_kc<256>(P, W, nraw, num_sms, st);
     if (need128 + 16 * 1024 <= 220 * 1024 && max_tasks <= 5120) return launch_kc<128>(P, W, nraw, num_sms, st);
     return launch_kc<64>(P, W, nraw, num_sms, st);
 }
