@@ -38,7 +38,7 @@ def _vals(n, p, rng, mode):
         elif r < 0.08:
             v = 0
         elif r < 0.12:
-            v = rng.randrange(2 ** 32)
+            v = rng.randrange(min(2 ** 32, M + 1))
         else:
             v = rng.randrange(M + 1)
         out.append(v if rng.random() < 0.5 else -v)
@@ -58,7 +58,7 @@ def _check(p1, p2, n, mode, seed, s1=3, s2=7):
 
 
 @pytest.mark.parametrize("p1,p2", [(90, 90), (200, 200), (300, 120), (305, 305), (500, 500), (1000, 1000),
-                                   (1300, 700), (700, 1300)])
+                                   (1300, 700), (700, 1300), (9, 1000), (1000, 9), (38, 300)])
 @pytest.mark.parametrize("n", [1, 129, 3001])
 def test_tc_contraction_shapes(p1, p2, n, monkeypatch):
     monkeypatch.setenv("UP_SPLIT", "1")
@@ -89,3 +89,21 @@ def test_tc_contraction_empty(monkeypatch):
             c.column_from_host_bin(200, 2, np.zeros((0, 21), np.uint32))]
     P, S, LA = c.sum_type("c1*c2", cols)
     assert up.result_to_string(c.sum_expr("c1*c2", cols), S) == up._fmt(0, S)
+
+
+def test_tc_two_products_and_signs(monkeypatch):
+    """two top-level products (two contractions sharing the workspace, one
+    negated) plus a rest term, vs exact Python"""
+    monkeypatch.setenv("UP_SPLIT", "1")
+    from paper_conf_icde_lixylz24_b200 import up
+    rng = random.Random(7)
+    n, p = 2500, 250
+    cols_v = [_vals(n, p, rng, "rand") for _ in range(4)]
+    c = up.Context(0)
+    cols = [c.column_from_host_bin(p, 0, *_words(v, p)) for v in cols_v]
+    expr = "c1*c2 - c3*c4 + c1"
+    P, S, LA = c.sum_type(expr, cols)
+    got = up.result_to_string(c.sum_expr(expr, cols), S)
+    c.check()
+    a, b, x, y = cols_v
+    assert got == up._fmt(sum(a[i] * b[i] - x[i] * y[i] + a[i] for i in range(n)), S)
