@@ -259,8 +259,11 @@ class ModexpWorkload(ExprWorkload):
     def roofline(self, kernel_ms, peaks):
         n = (self.N.bit_length() + 31) // 32
         montmuls = (self.e.bit_length() - 1) + bin(self.e).count("1") - 1 + 2   # squarings + multiplies + in/out
-        return self._alu_roofline(kernel_ms, montmuls * (2 * n * n + n),
-                                  f"; {montmuls} Montgomery products x (2n^2+n), n = {n}")
+        note = f"; {montmuls} Montgomery products x (2n^2+n), n = {n} (SURVEY §8d count)"
+        if self.e % 2 == 1 and self.e > 1 and n <= 40:
+            note += ("; the radix-2^28 kernel performs one fewer: for odd e its last multiply takes the plain base "
+                     "and leaves Montgomery form")
+        return self._alu_roofline(kernel_ms, montmuls * (2 * n * n + n), note)
 
     def oracle_sum(self, ocols, n, threads):
         import oracle
