@@ -260,7 +260,7 @@ class ModexpWorkload(ExprWorkload):
         n = (self.N.bit_length() + 31) // 32
         montmuls = (self.e.bit_length() - 1) + bin(self.e).count("1") - 1 + 2   # squarings + multiplies + in/out
         note = f"; {montmuls} Montgomery products x (2n^2+n), n = {n} (SURVEY §8d count)"
-        if self.e % 2 == 1 and self.e > 1 and n <= 40:
+        if self.e % 2 == 1 and self.e > 1 and n <= 64:
             note += ("; the radix-2^28 kernel performs one fewer: for odd e its last multiply takes the plain base "
                      "and leaves Montgomery form")
         return self._alu_roofline(kernel_ms, montmuls * (2 * n * n + n), note)
