@@ -261,8 +261,8 @@ class ModexpWorkload(ExprWorkload):
         montmuls = (self.e.bit_length() - 1) + bin(self.e).count("1") - 1 + 2   # squarings + multiplies + in/out
         note = f"; {montmuls} Montgomery products x (2n^2+n), n = {n} (SURVEY §8d count)"
         if self.e % 2 == 1 and self.e > 1 and n <= 64:
-            note += ("; the radix-2^28 kernel performs one fewer: for odd e its last multiply takes the plain base "
-                     "and leaves Montgomery form")
+            note += ("; the radix-2^28 kernel performs up to two fewer: for odd e its last multiply takes the plain "
+                     "base and leaves Montgomery form, and the base's zero upper chunk (x < R) needs no conversion product")
         return self._alu_roofline(kernel_ms, montmuls * (2 * n * n + n), note)
 
     def oracle_sum(self, ocols, n, threads):
