@@ -257,6 +257,39 @@ def test_brute_force_expressions(expr):
         assert len(got.split(".")[1]) == S if S else "." not in got
 
 
+@pytest.mark.parametrize("terms", [2, 3, 5, 8, 11])
+def test_query5_literal_brute_force(terms):
+    """Paper-literal Query 5 (the SQL Taylor polynomial of sin
+    with 2..11 terms over DECIMAL(9,8) x): the oracle's rows equal the exact
+    rational evaluation with the paper's per-division truncation (brute_eval),
+    and every row lies within the truncation budget of the exact polynomial
+    sum_k (-1)^k x^(2k+1)/(2k+1)!: term k's division truncates at scale
+    8(2k+1)+4, so |row - poly| < sum_k 10^-(8(2k+1)+4); with 11
+    terms the polynomial is within x^23/23! (+ float rounding) of sin x."""
+    rng = random.Random(terms)
+    xs = []
+    for mu in (0.01, 0.78, 1.56):
+        mag, neg = synth.normal_decimal(12, mu, 0.01, 8, config=5, column=3)
+        xs += [(-int(m[0]) if g else int(m[0])) for m, g in zip(mag, neg)]
+    xs += [0, 1, -1, 10 ** 9 - 1, -(10 ** 9 - 1), rng.randrange(10 ** 9)]
+    vals = [_fmt(m, 8) for m in xs]
+    e = "c1"
+    for k in range(1, terms):
+        n = 2 * k + 1
+        e += (" - " if k % 2 else " + ") + "*".join(["c1"] * n) + "/" + str(math.factorial(n))
+    col = Column(9, 8, strings=vals)
+    got = oracle.eval_rows(e, [col])
+    P, S = oracle.expr_type(e, [col])
+    for v, g in zip(vals, got):
+        want, ws = brute_eval(e, [(9, 8)], [v])
+        assert ws == S and dec(g) == want, (terms, v, g, want)
+        x = Fraction(v)
+        poly = sum(Fraction((-1) ** k) * x ** (2 * k + 1) / math.factorial(2 * k + 1) for k in range(terms))
+        assert abs(dec(g) - poly) < sum(Fraction(1, 10 ** (8 * (2 * k + 1) + 4)) for k in range(1, terms))
+        if terms == 11:
+            assert abs(poly - Fraction(math.sin(float(x)))) <= abs(x) ** 23 / math.factorial(23) + Fraction(1, 10 ** 15)
+
+
 def test_modulo_brute_force():
     rng = random.Random(7)
     for _ in range(300):
