@@ -486,7 +486,7 @@ def main():
         for i in range(K):
             if flush is not None:
                 flush.zero_()            # evict the inputs from L2 (outside the step's events)
-                torch.sum(flush_rd, out=flush_sum)
+                torch.sum(flush_rd, dim=0, out=flush_sum)
             sev[i][0].record(stream)
             kev[i][0].record(stream)
             wl.kernel(partial)

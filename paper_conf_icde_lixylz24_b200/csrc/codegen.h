@@ -62,6 +62,6 @@ struct ModexpPlan {
 };
 std::string gen_modexp_kernel(const HBig &N, const HBig &e, const ModexpPlan &plan, bool sum, std::string &err);
 std::string gen_sin_kernel(int P, int p, int s, int Lx, int Lout, int LA, bool sum, int &lanes_per_row, std::string &err,
-                           int *smem_per_thread = nullptr);
+                           int *smem_per_thread = nullptr, bool *is_v3 = nullptr);
 
 }  // namespace uph
