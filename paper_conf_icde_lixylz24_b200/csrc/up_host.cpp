@@ -1171,9 +1171,12 @@ up_status up_internal_compile(up_ctx *c, const std::string &src, int rows_per_th
         k->threads = threads;
         if (dyn_smem > 0)
             CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, dyn_smem));
+        if (const char *cv = getenv("UP_SMEM_CARVEOUT"))   // measurement knob: preferred shared-memory carveout (%)
+            CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, atoi(cv)));
         k->dyn_smem = dyn_smem;
         int nb = 0;
         CU_TRY(drv.OccupancyMaxActiveBlocksPerMultiprocessor(&nb, k->fn, threads, (size_t)dyn_smem));
+        if (getenv("UP_PRINT_OCC")) fprintf(stderr, "[libup] %d threads, %d B dynamic smem: %d blocks/SM\n", threads, dyn_smem, nb);
         k->blocks_per_sm = std::max(1, nb);
     }
     *fn_out = k;
