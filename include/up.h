@@ -207,8 +207,9 @@ up_status up_filter(up_ctx *ctx, const char *lhs, const char *op, const char *rh
  * DeviceRadixSort, one pass per 32-bit limb, least significant key column
  * and limb first, the top limb's sign bit flipped so two's complement orders
  * as signed; excluded rows sorted last), an adjacent-difference pass over all
- * limbs, a prefix sum and a scatter.  Scratch: ~20 bytes per row
- * (stream-ordered allocations).
+ * limbs, a prefix sum and a scatter.  Scratch: the ctx's persistent scratch
+ * buffer (24 bytes per row + sort temporaries), grown on demand (growing it
+ * synchronises the device); the call holds the ctx lock throughout.
  */
 up_status up_group_ids(up_ctx *ctx, const up_column *keys, int nkeys, int32_t *d_ids, int64_t *n_groups,
                        int64_t *d_first, void *stream);

@@ -11,6 +11,7 @@
 #include <cuda_runtime.h>
 
 #include <cub/cub.cuh>
+#include <mutex>
 #include <string>
 
 #include "../../include/up.h"
@@ -18,6 +19,7 @@
 up_status up_internal_fail(up_status st, const std::string &msg);
 void up_internal_add_launches(up_ctx *c, long long k);
 up_status up_internal_scratch(up_ctx *c, size_t bytes, void **out);
+std::mutex &up_internal_mutex(up_ctx *c);
 
 namespace {
 
@@ -105,13 +107,21 @@ extern "C" up_status up_group_ids(up_ctx *c, const up_column *keys, int nkeys, i
     *n_groups = 0;
     if (n == 0) return UP_OK;
     cudaStream_t st = (cudaStream_t)stream;
+    // the ctx scratch may be reallocated by up_internal_scratch: hold the ctx lock for the whole call
+    std::lock_guard<std::mutex> lock(up_internal_mutex(c));
+#define GB_TRY(x)                                                                                     \
+    do {                                                                                              \
+        const cudaError_t e_ = (x);                                                                   \
+        if (e_ != cudaSuccess) return up_internal_fail(UP_E_CUDA, std::string("group_ids: " #x ": ") + \
+                                                       cudaGetErrorString(e_));                       \
+    } while (0)
     // scratch (the ctx's persistent buffer): keys x2, perm x2, head, gid, then CUB's temp storage
     uint32_t *k0 = nullptr;
     size_t tsort = 0, tscan = 0;
     {
         cub::DoubleBuffer<uint32_t> kq(nullptr, nullptr), pq(nullptr, nullptr);
-        cub::DeviceRadixSort::SortPairs(nullptr, tsort, kq, pq, n, 0, 32, st);
-        cub::DeviceScan::InclusiveSum(nullptr, tscan, (uint32_t *)nullptr, (uint32_t *)nullptr, n, st);
+        GB_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tsort, kq, pq, n, 0, 32, st));
+        GB_TRY(cub::DeviceScan::InclusiveSum(nullptr, tscan, (uint32_t *)nullptr, (uint32_t *)nullptr, n, st));
     }
     const size_t tbytes = tsort > tscan ? tsort : tscan;
     const size_t words = ((6 * (size_t)n + 63) / 64) * 64;
@@ -133,28 +143,29 @@ extern "C" up_status up_group_ids(up_ctx *c, const up_column *keys, int nkeys, i
             k_gb_gather<<<grid, 256, 0, st>>>(col.data + (long long)j * col.ld, pb.Current(), kb.Current(), n, flip);
             ++launches;
             size_t tb = tbytes;
-            cub::DeviceRadixSort::SortPairs(temp, tb, kb, pb, n, 0, 32, st);
+            GB_TRY(cub::DeviceRadixSort::SortPairs(temp, tb, kb, pb, n, 0, 32, st));
         }
     }
     k_gb_gather_excl<<<grid, 256, 0, st>>>(d_ids, pb.Current(), kb.Current(), n);
     ++launches;
     {
         size_t tb = tbytes;
-        cub::DeviceRadixSort::SortPairs(temp, tb, kb, pb, n, 0, 1, st);
+        GB_TRY(cub::DeviceRadixSort::SortPairs(temp, tb, kb, pb, n, 0, 1, st));
     }
     k_gb_heads<<<grid, 256, 0, st>>>(kp, d_ids, pb.Current(), head, n);
     ++launches;
     {
         size_t tb = tbytes;
-        cub::DeviceScan::InclusiveSum(temp, tb, head, gid, n, st);
+        GB_TRY(cub::DeviceScan::InclusiveSum(temp, tb, head, gid, n, st));
     }
     uint32_t total = 0;
-    cudaMemcpyAsync(&total, gid + (n - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st);
+    GB_TRY(cudaMemcpyAsync(&total, gid + (n - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
     k_gb_scatter<<<grid, 256, 0, st>>>(pb.Current(), head, gid, d_ids, reinterpret_cast<long long *>(d_first), n);
     ++launches;
     up_internal_add_launches(c, launches);
-    const cudaError_t e = cudaStreamSynchronize(st);
-    if (e != cudaSuccess) return up_internal_fail(UP_E_CUDA, std::string("group_ids: ") + cudaGetErrorString(e));
+    GB_TRY(cudaGetLastError());
+    GB_TRY(cudaStreamSynchronize(st));
+#undef GB_TRY
     *n_groups = (int64_t)total;
     return UP_OK;
 }

@@ -522,8 +522,13 @@ up_status up_column_from_host_bin(up_ctx *c, const uint32_t *mag, int32_t W, con
         CUDA_TRY(cudaMemcpyAsync(c->d_stage, mag, mb, cudaMemcpyHostToDevice, st));
         if (neg) CUDA_TRY(cudaMemcpyAsync((char *)c->d_stage + mb_al, neg, nb, cudaMemcpyHostToDevice, st));
     }
-    return up_column_from_device_bin(c, (const uint32_t *)c->d_stage, W,
-                                     neg ? (const uint8_t *)((char *)c->d_stage + mb_al) : nullptr, dst, stream);
+    if (up_status s = up_column_from_device_bin(c, (const uint32_t *)c->d_stage, W,
+                                                neg ? (const uint8_t *)((char *)c->d_stage + mb_al) : nullptr, dst,
+                                                stream))
+        return s;
+    // up.h: the caller may reuse or free the host buffers when this returns
+    CUDA_TRY(cudaStreamSynchronize(st));
+    return UP_OK;
 }
 
 up_status up_column_from_host(up_ctx *c, const char *const *decimals, up_column *dst, void *stream) {
@@ -590,7 +595,9 @@ up_status up_column_from_host_compact(up_ctx *c, const uint8_t *bytes, up_column
         if (up_status s = ensure_stage(c, nb, st)) return s;
         CUDA_TRY(cudaMemcpyAsync(c->d_stage, bytes, nb, cudaMemcpyHostToDevice, st));
     }
-    return up_column_from_device_compact(c, (const uint8_t *)c->d_stage, dst, stream);
+    if (up_status s = up_column_from_device_compact(c, (const uint8_t *)c->d_stage, dst, stream)) return s;
+    CUDA_TRY(cudaStreamSynchronize(st));   // up.h: host buffer reusable on return
+    return UP_OK;
 }
 
 up_status up_column_to_host_compact(up_ctx *c, const up_column *col, uint8_t *bytes, void *stream) {

@@ -46,5 +46,25 @@ def gpu_sum_string(expr, gcols, n_global=0):
 
 
 def int_rows_to_strings(vals, s):
-    from paper_conf_icde_lixylz24_b200.up import _fmt
-    return [_fmt(v, s) for v in vals]
+    """Mantissas at scale s -> "[-]int.frac" input strings (test-local)."""
+    out = []
+    for v in vals:
+        a = str(abs(v))
+        if s:
+            a = a.rjust(s + 1, "0")
+            a = a[:-s] + "." + a[-s:]
+        out.append(("-" if v < 0 else "") + a)
+    return out
+
+
+def limbs_int(limb_tensor) -> int:
+    """Two's-complement little-endian 32-bit limbs (device tensor or list) ->
+    Python int, written here so expected values never pass through libup's
+    own formatter or converters."""
+    vals = limb_tensor.detach().cpu().tolist() if hasattr(limb_tensor, "detach") else list(limb_tensor)
+    v = 0
+    for x in reversed(vals):
+        v = (v << 32) | (int(x) & 0xFFFFFFFF)
+    if vals and int(vals[-1]) & 0x80000000:
+        v -= 1 << (32 * len(vals))
+    return v

@@ -111,12 +111,22 @@ def test_sum_expr_parity(case, n):
     expr, types = case
     host = G.gen_cols(n, types, nonzero_lead_cols=_lead(expr, types))
     ocols = G.to_oracle(host, types)
+    gcols = G.to_gpu(host, types) if n else [G.ctx().column_from_host_bin(p, s, np.zeros((0, 1), np.uint32))
+                                             for p, s in types]
     try:
         want, P, S = oracle.eval_sum(expr, ocols, n=n, threads=4)
     except oracle.OracleError as e:
-        pytest.skip(f"oracle flags {e.name} for this seed")
-    gcols = G.to_gpu(host, types) if n else [G.ctx().column_from_host_bin(p, s, np.zeros((0, 1), np.uint32))
-                                             for p, s in types]
+        # a row the oracle rejects (÷0 / overflow of the typed quotient, readings
+        # Q5/Q6) must raise the same sticky flag on the GPU
+        from paper_conf_icde_lixylz24_b200.up import UpError
+        c = G.ctx()
+        c.sum_expr(expr, gcols)
+        with pytest.raises(UpError) as ei:
+            c.check()
+        rows = oracle.eval_rows(expr, ocols, n=n, strict=False)
+        raised = {oracle.STATUS[int(w[1:])] for w in rows if w.startswith("E")} or {e.name}
+        assert ei.value.name in raised, (ei.value.name, raised)
+        return
     got, gP, gS = G.gpu_sum_string(expr, gcols)
     assert (gP, gS) == (P, S)
     assert got == want

@@ -15,7 +15,7 @@ def _x(n, mu, col=1):
     return synth.normal_decimal(n, mu, 0.01, 8, config=5, column=col)
 
 
-@pytest.mark.parametrize("P,n", [(8, 300), (20, 300), (60, 300), (100, 200), (500, 40), (1000, 12), (5000, 3)])
+@pytest.mark.parametrize("P,n", [(8, 300), (20, 300), (60, 300), (100, 200), (500, 130), (1000, 40), (5000, 40)])
 @pytest.mark.parametrize("mu", [0.01, 0.78, 1.56])
 def test_sin_rows_parity(P, n, mu):
     mag, neg = _x(n, mu)
@@ -28,8 +28,9 @@ def test_sin_rows_parity(P, n, mu):
     assert got == want
 
 
-def test_sin_20000_digits_sampled():
-    mag, neg = _x(2, 0.78)
+def test_sin_20000_digits_rows():
+    """32-lane groups, 8 rows per 256-thread block: 10 rows = one full block + a ragged one"""
+    mag, neg = _x(10, 0.78)
     c = G.ctx()
     out = c.sin_taylor(c.column_from_host_bin(9, 8, mag, neg), 20000)
     c.check()
@@ -57,8 +58,12 @@ def test_sin_edge_inputs(p, s, vals):
         assert c.column_to_strings(out) == oracle.sin_rows(oracle.Column(p, s, strings=vals), P), (p, s, P)
 
 
-@pytest.mark.parametrize("P,n", [(30, 5000), (500, 300), (2000, 40)])
+@pytest.mark.parametrize("P,n", [(30, 5000), (500, 300), (2000, 40), (5000, 70), (20000, 17)])
 def test_sin_sum_parity(P, n):
+    """Fused SUM(sin_P) vs the oracle in every kernel regime: one row per
+    thread (P <= ~1800), 8-lane groups (P = 5000: 32 rows per block, 70 rows =
+    two full blocks + a ragged third) and 32-lane groups (P = 20000: 8 rows per
+    block, 17 rows = two full blocks + one row)."""
     mag, neg = _x(n, 0.78, col=2)
     c = G.ctx()
     res = c.sin_taylor_sum(c.column_from_host_bin(9, 8, mag, neg), P)

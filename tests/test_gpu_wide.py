@@ -1,6 +1,14 @@
-"""GPU parity of the wide SUM regime (warp per row, rows a10/a11): cfg3's
-SUM(c1*c2 - c3/c4) at DECIMAL(200,50) / (500,75) / (1000,100) and other
-linear combinations of column, product and quotient terms, vs the oracle."""
+"""GPU parity of SUMs over wide numbers (rows a6/a7/a10/a11) vs the oracle.
+
+Which kernel runs (up_host.cpp::expr_kernel / up_sum_expr):
+* top-level column products of a SUM take the tensor-core row contraction
+  (contract_tc.cu) and the rest runs in the per-thread fused kernel (one row
+  per thread, up to 256 limbs) -- cfg3 at DECIMAL(200,50) / (500,75) /
+  (1000,100) and the linear combinations below;
+* numbers of >= 257 limbs (p >= ~2470 digits) take the warp-per-row wide
+  regime (up_wide.cuh, codegen.cpp::gen_wide_sum_kernel): a warp owns one
+  row, operands staged in shared memory -- test_warp_per_row_* below reach it
+  (the kernel source is checked to be the wide one)."""
 import os
 
 import numpy as np
@@ -57,26 +65,6 @@ def test_wide_edge_values_and_flags():
     with pytest.raises(up.UpError) as ei:
         c.check()
     assert ei.value.name in ("DIVZERO", "OVERFLOW")
-
-
-def test_wide_and_per_thread_paths_agree(monkeypatch):
-    """p=200 sits on the regime boundary: the per-thread fused kernel
-    (UP_NO_WIDE) and the wide kernel must give the same bits."""
-    types = [(200, 50)] * 4
-    host = G.gen_cols(500, types, config=3, nonzero_lead_cols=(3,), seed=7)
-    from paper_conf_icde_lixylz24_b200 import up
-    c1 = up.Context(0)
-    a, _, _ = (None, None, None)
-    cols = [c1.column_from_host_bin(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
-    P, S, LA = c1.sum_type("c1*c2 - c3/c4", cols)
-    wide = up.result_to_string(c1.sum_expr("c1*c2 - c3/c4", cols), S)
-    c1.check()
-    monkeypatch.setenv("UP_NO_WIDE", "1")
-    c2 = up.Context(0)
-    cols2 = [c2.column_from_host_bin(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
-    narrow = up.result_to_string(c2.sum_expr("c1*c2 - c3/c4", cols2), S)
-    c2.check()
-    assert wide == narrow
 
 
 @pytest.mark.parametrize("expr,types,lead", [
@@ -141,7 +129,50 @@ def test_split_contraction_extreme_values(p, radix, monkeypatch):
     c = up.Context(0)
     cols = [c.column_from_host_bin(p, 10, *words(vals1)), c.column_from_host_bin(p, 10, *words(vals2))]
     P, S, LA = c.sum_type("c1*c2", cols)
-    got = up.result_to_string(c.sum_expr("c1*c2", cols), S)
+    got = G.limbs_int(c.sum_expr("c1*c2", cols))
     c.check()
-    want = sum(a * b for a, b in zip(vals1, vals2))
-    assert got == up._fmt(want, S)
+    assert got == sum(a * b for a, b in zip(vals1, vals2))   # mantissas at scale S
+
+
+def _wide_source(expr, types, n):
+    from paper_conf_icde_lixylz24_b200 import up
+    return up.gen_source("sum", expr, types, n)
+
+
+@pytest.mark.parametrize("expr,types,lead,env", [
+    ("c1+c2", [(2500, 10), (2480, 300)], (), None),
+    ("c1 - c2 + c1", [(2600, 0), (2600, 0)], (), None),
+    ("c1/c2 - c3", [(2500, 0), (30, 0), (2490, 4)], (1,), None),
+    ("-c1/c2 + c3/c4", [(2550, 20), (700, 10), (2520, 3), (20, 1)], (1, 3), None),
+    ("c1*c2 - c3", [(1300, 5), (1250, 7), (2000, 12)], (), "UP_NO_SPLIT"),
+])
+@pytest.mark.parametrize("n", [1, 9, 300])
+def test_warp_per_row_wide_regime_parity(expr, types, lead, env, n, monkeypatch):
+    """>= 257-limb SUM terms: the warp-per-row kernel (up_wide.cuh) vs the oracle."""
+    if env:
+        monkeypatch.setenv(env, "1")
+    assert "wide SUM regime" in _wide_source(expr, types, n)
+    got, want = _sum(expr, types, n, lead=lead, seed=n + 5)
+    assert got == want
+
+
+def test_warp_per_row_wide_regime_extremes():
+    """all-nines magnitudes with mixed signs (full carry ripple through 270
+    limbs) and a divide-by-zero row raising the sticky flag"""
+    from paper_conf_icde_lixylz24_b200 import up
+    c = G.ctx()
+    p = 2600
+    big = str(10 ** p - 1)
+    v1 = [big, "-" + big, big, "0", "1", big, "-1"]
+    v2 = [big, big, "-" + big, big, "-" + big, "0", "-1"]
+    assert "wide SUM regime" in _wide_source("c1 - c2 + c1", [(p, 0), (p, 0)], len(v1))
+    g = [c.column_from_strings(p, 0, v1), c.column_from_strings(p, 0, v2)]
+    o = [oracle.Column(p, 0, strings=v1), oracle.Column(p, 0, strings=v2)]
+    res = c.sum_expr("c1 - c2 + c1", g)
+    c.check()
+    assert up.result_to_string(res, 0) == oracle.eval_sum("c1 - c2 + c1", o)[0]
+    d = [c.column_from_strings(p, 0, v1), c.column_from_strings(20, 0, ["7", "3", "0", "1", "9", "2", "5"])]
+    c.sum_expr("c1/c2", d)
+    with pytest.raises(up.UpError) as ei:
+        c.check()
+    assert ei.value.name == "DIVZERO"

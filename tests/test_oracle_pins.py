@@ -469,3 +469,48 @@ def test_sin_small_P_matches_decimal_context():
         t = -t * x * x / ((2 * k) * (2 * k + 1)); k += 1
     got = decimal.Decimal(oracle.sin_rows(Column(9, 8, strings=["0.50000000"]), 20)[0])
     assert abs(got - s) <= decimal.Decimal(10) ** -20 * 12
+
+
+def _sin_q13_python(m: int, s: int, P: int) -> str:
+    """Reading Q13 written out with Python ints, term by
+    term in the order the definition states: t_1 = |m| 10^(P-s),
+    t_(k+1) = floor(t_k m^2 / (10^(2s) (2k)(2k+1))), stop at t = 0,
+    S = sum (-1)^(k-1) t_k, result sign(m) S at scale P.  Independent of
+    oracle/updec.c (base-10^9 C); the canonical string has exactly P fraction
+    digits and no "-0"."""
+    t, k, S = abs(m) * 10 ** (P - s), 1, 0
+    while t:
+        S += t if k % 2 == 1 else -t
+        t = t * m * m // (10 ** (2 * s) * (2 * k) * (2 * k + 1))
+        k += 1
+    v = -S if m < 0 else S
+    sign = "-" if v < 0 else ""
+    a = str(abs(v)).rjust(P + 1, "0")
+    return sign + a[:-P] + "." + a[-P:]
+
+
+@pytest.mark.parametrize("P", [8, 57, 300, 1000])
+@pytest.mark.parametrize("mu", [0.01, 0.78, 1.56])
+@pytest.mark.parametrize("s", [0, 2, 8])
+def test_sin_bits_match_q13_python_int_brute_force(P, mu, s):
+    """Pins the BITS of oracle.sin_rows (the accuracy tests above pin only the
+    value to within (K+1) ulps): a floor->round or floor->ceil slip, a dropped
+    term or a wrong sign in the recurrence fails here.  Query 5's inputs are
+    x ~ N(mu, 0.01^2) with mu in {0.01, 0.78, 1.56} (§IV, reading
+    Q14), here rounded to scale s in {0, 2, 8} (p = s + 1 digits, |x| < 10)."""
+    n = 25
+    mag, neg = synth.normal_decimal(n, mu, 0.01, s, config=5, column=7)
+    col = Column(s + 1, s, mag, neg)
+    got = oracle.sin_rows(col, P)
+    want = [_sin_q13_python(m, s, P) for m in synth.to_ints(mag, neg)]
+    assert got == want
+
+
+def test_sin_bits_q13_edge_values():
+    """Boundary mantissas: zero, one ulp, the largest DECIMAL(9,8) magnitude
+    (|x| just below 10), and negative values."""
+    vals = ["0", "0.00000001", "-0.00000001", "9.99999999", "-9.99999999", "3.14159265", "-1.57079633"]
+    ms = [int(v.replace(".", "")) for v in vals]
+    for P in (8, 40, 333):
+        got = oracle.sin_rows(Column(9, 8, strings=vals), P)
+        assert got == [_sin_q13_python(m, 8, P) for m in ms], P
