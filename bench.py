@@ -32,6 +32,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+E2E_MAX_ROWS = 1 << 26
 METRIC = "tuples/sec for SELECT SUM(expr) by DECIMAL precision at 1/2/4/8 B200; % HBM/INT peak"
 # Integer roofline for the compute-bound configs, in 32x32->64 LIMB PRODUCTS/s.
 # Every limb product needs one high-half multiply (IMAD.HI / the high half of
@@ -57,6 +58,12 @@ CONFIGS = {
     5: dict(kind="sin", name="cfg5 SUM(sin_P(x)) P=1000, x~N(0.78,0.01) DECIMAL(9,8)", P=1000, mu=0.78,
             rows=1_000_000),
 }
+
+
+def traffic_key(cfg, rows):
+    """profiles/traffic/<key>.json key: the workload name + rows per GPU."""
+    import re
+    return re.sub(r"[^A-Za-z0-9]+", "_", cfg["name"]).strip("_") + f"_{rows}"
 
 
 def _peaks():
@@ -130,6 +137,9 @@ class Workload:
     def __init__(self, cfg, args, ctx, rows, n_global, row0):
         self.cfg, self.args, self.ctx = cfg, args, ctx
         self.rows, self.n_global, self.row0 = rows, n_global, row0
+        # e2e (host buffers -> result) runs on at most E2E_MAX_ROWS of this
+        # rank's rows: pinned host copies of 2^30-row columns would be 15-31 GB
+        self.e2e_rows = min(rows, E2E_MAX_ROWS)
 
 
 class ExprWorkload(Workload):
@@ -145,7 +155,7 @@ class ExprWorkload(Workload):
             self.cols.append(ctx.column_from_device_bin(p, s, mag, neg))
         ctx.check()
         self.P, self.S, self.LA = ctx.sum_type(cfg["expr"], self.cols, self.n_global)
-        self.e2e_cols = [up.Column(p, s, self.rows) for p, s in cfg["types"]]
+        self.e2e_cols = [up.Column(p, s, self.e2e_rows) for p, s in cfg["types"]]
         self.bytes_per_row = sum(4 * up.limbs(p) for p, s in cfg["types"])
 
     def kernel(self, out):
@@ -159,7 +169,8 @@ class ExprWorkload(Workload):
         from gen import synth
         bufs = []
         for (mag, neg), (p, s) in zip(self.raw, self.cfg["types"]):
-            cb = synth.to_compact(mag.cpu().numpy().view(np.uint32), neg.cpu().numpy(), p)
+            m, g = mag[: self.e2e_rows], neg[: self.e2e_rows]
+            cb = synth.to_compact(m.cpu().numpy().view(np.uint32), g.cpu().numpy(), p)
             t = torch.empty(cb.shape, dtype=torch.uint8, pin_memory=True)
             t.copy_(torch.from_numpy(cb))
             bufs.append(t)
@@ -167,7 +178,7 @@ class ExprWorkload(Workload):
 
     def e2e_ingest(self, host):
         for hb, (p, s), col in zip(host, self.cfg["types"], self.e2e_cols):
-            self.ctx.column_from_compact(p, s, hb, n=self.rows, out=col)
+            self.ctx.column_from_compact(p, s, hb, n=self.e2e_rows, out=col)
 
     def e2e_kernel(self, out):
         self.ctx.sum_expr(self.cfg["expr"], self.e2e_cols, self.n_global, out=out)
@@ -215,10 +226,12 @@ class ExprWorkload(Workload):
                 "alg_unit": f"{products_per_row} 32x32->64 limb products/row x {self.rows} rows" + note,
                 "peak_source": src}
 
-    def host_for_oracle(self):
+    def host_for_oracle(self, max_rows=1 << 25):
+        """Host copies of (at most the first max_rows of) the inputs for the oracle."""
         import numpy as np
         import oracle
-        return [oracle.Column(p, s, m.cpu().numpy().view(np.uint32), g.cpu().numpy())
+        k = min(self.rows, max_rows)
+        return [oracle.Column(p, s, m[:k].cpu().numpy().view(np.uint32), g[:k].cpu().numpy())
                 for (m, g), (p, s) in zip(self.raw, self.cfg["types"])]
 
     def oracle_sum(self, ocols, n, threads):
@@ -247,7 +260,7 @@ class ModexpWorkload(ExprWorkload):
         ctx.check()
         self.P, self.LA = ctx.modexp_sum_type(self.N, self.n_global)
         self.S = 0
-        self.e2e_cols = [up.Column(self.d, 0, self.rows)]
+        self.e2e_cols = [up.Column(self.d, 0, self.e2e_rows)]
         self.cfg = dict(cfg, types=[(self.d, 0)])
 
     def kernel(self, out):
@@ -291,7 +304,7 @@ class SinWorkload(ExprWorkload):
         self.P = up.sum_precision(self.Pd + 1, self.n_global)
         self.S = self.Pd
         self.LA = up.limbs(self.P)
-        self.e2e_cols = [up.Column(9, 8, self.rows)]
+        self.e2e_cols = [up.Column(9, 8, self.e2e_rows)]
         self.cfg = dict(cfg, types=[(9, 8)])
         # active-limb sum per row, from a sample of rows
         import numpy as np
@@ -335,19 +348,21 @@ def cpu_baseline(wl, budget_s=12.0):
     host cores (pthreads, static row blocks, exact combine)."""
     cores = len(os.sched_getaffinity(0))
     ocols = wl.host_for_oracle()
-    n_all = ocols[0].n
+    n_all = ocols[0].n          # <= wl.rows (the copy is capped for 2^30-row columns)
     n = min(n_all, 64)
     t0 = time.perf_counter()
-    wl.oracle_sum(ocols, n, cores)
+    val = wl.oracle_sum(ocols, n, cores)
     dt = time.perf_counter() - t0
     while dt < budget_s / 8 and n < n_all:
         n = int(min(n_all, n * max(2.0, budget_s / 2 / max(dt, 1e-4))))
         t0 = time.perf_counter()
-        wl.oracle_sum(ocols, n, cores)
+        val = wl.oracle_sum(ocols, n, cores)
         dt = time.perf_counter() - t0
-    return {"value": n / dt, "unit": "tuples/s", "cores": cores, "kind": "oracle",
-            "sample": f"first {n} of {n_all} rows of the same seeded workload ({wl.cfg['name']}), "
-                      f"{cores} threads, {dt:.2f} s"}
+    out = {"value": n / dt, "unit": "tuples/s", "cores": cores, "kind": "oracle",
+           "sample": f"first {n} of {n_all} rows of the same seeded workload ({wl.cfg['name']}), "
+                     f"{cores} threads, {dt:.2f} s"}
+    # the oracle's SUM over every row is the parity check of the bench's own result
+    return out, (val if n == wl.rows else None)
 
 
 def run_reference(args, cfg):
@@ -404,6 +419,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", type=int, default=2)
     ap.add_argument("--rows", type=int, default=0, help="rows per GPU (default: the config's)")
+    ap.add_argument("--global-rows", type=int, default=0, help="total rows, sharded over the GPUs (strong scaling)")
     ap.add_argument("--impl", default="up", choices=["up", "reference"])
     ap.add_argument("--ref-rows", type=int, default=200_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -438,6 +454,7 @@ def main():
 
     from gen import device as gdev
     from paper_conf_icde_lixylz24_b200 import up
+    from paper_conf_icde_lixylz24_b200.dist import ShardedSum, shard_range
 
     ws, rank, local = dist_env()
     torch.cuda.set_device(local)
@@ -445,15 +462,27 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     ctx = up.Context(local)
     stream = torch.cuda.current_stream()
-    rows = args.rows or cfg["rows"]
-    n_global = rows * ws
+    # Row sharding (rows a13/e).  N = 1: the config's rows (configs[1]:
+    # 10M).  N > 1, memory-bound configs 1/2: STRONG scaling of 2^30-row columns
+    # (SURVEY §8e), so the all-gather + combine stays a small part of the step;
+    # compute-bound configs 3-5: weak scaling (the config's rows per GPU).
+    # --global-rows / --rows override.
+    if args.global_rows:
+        n_global, scaling = args.global_rows, "strong"
+    elif ws > 1 and cfg["kind"] == "expr" and cfg["types"][0][0] < 100 and not args.rows:
+        n_global, scaling = 1 << 30, "strong"
+    else:
+        n_global, scaling = (args.rows or cfg["rows"]) * ws, "weak"
+    lo, hi = shard_range(n_global, ws, rank)
+    rows = hi - lo
     gdev.build()
-    wl = KINDS[cfg["kind"]](cfg, args, ctx, rows, n_global, rank * rows)
+    wl = KINDS[cfg["kind"]](cfg, args, ctx, rows, n_global, lo)
     wl.setup()
     LA = wl.LA
-    partial = torch.empty(LA, dtype=torch.int32, device="cuda")
-    gathered = torch.empty(LA * ws, dtype=torch.int32, device="cuda")
-    total = torch.empty(LA, dtype=torch.int32, device="cuda")
+    # one pass of the hot path = the rank's fused SUM kernel, then (N > 1) the
+    # NCCL all-gather of the LA-limb partials and the exact combine kernel
+    ss = ShardedSum(ctx, LA, wl.S, wl.kernel)
+    partial = ss.partial
     # L2 flush buffer for working sets below L2 (cfg1: 16 MB)
     flush = None
     if getattr(wl, "bytes_per_row", 0) * rows < 256e6 and cfg["kind"] == "expr" and cfg["types"][0][0] < 100:
@@ -464,10 +493,7 @@ def main():
         flush_sum = torch.empty((), dtype=torch.float32, device="cuda")
 
     def step():
-        wl.kernel(partial)
-        if ws > 1:
-            dist.all_gather_into_tensor(gathered, partial)
-            ctx.sum_combine(gathered, LA, out=total)
+        ss()
 
     for _ in range(max(3, args.warmup)):     # warm-up (includes the one-time specialisation / JIT)
         step()
@@ -491,9 +517,9 @@ def main():
             kev[i][0].record(stream)
             wl.kernel(partial)
             kev[i][1].record(stream)
-            if ws > 1:
-                dist.all_gather_into_tensor(gathered, partial)
-                ctx.sum_combine(gathered, LA, out=total)
+            if ws > 1:     # the exchange step of ShardedSum.__call__ (split out to time the kernel alone)
+                dist.all_gather_into_tensor(ss.gathered, partial)
+                ctx.sum_combine(ss.gathered, LA, out=ss.total)
             sev[i][1].record(stream)
         torch.cuda.synchronize()
     if ws > 1:
@@ -508,14 +534,21 @@ def main():
     ms_per_step = ms / K
     value = n_global / (ms_per_step / 1e3)
     ctx.check()
-    result = up.result_to_string(total if ws > 1 else partial, wl.S)
+    result = ss.result()
     peaks = _peaks()
     roofline = wl.roofline(kernel_ms, peaks)
-    tp = os.path.join(ROOT, "profiles", f"traffic_cfg{args.config}.json")
+    # traffic = dram__bytes_read + dram__bytes_write of the dominant kernel per
+    # launch, from one `ncu --set full` capture of THIS workload (same config,
+    # precision and rows per GPU), summarised by tools/ncu_summary.py
+    tkey = traffic_key(cfg, rows)
+    tp = os.path.join(ROOT, "profiles", "traffic", f"{tkey}.json")
     roofline["traffic"] = None
+    roofline["traffic_key"] = tkey
     if os.path.exists(tp):
         try:
-            roofline["traffic"] = json.load(open(tp)).get("dram_bytes_per_launch")
+            t = json.load(open(tp))
+            roofline["traffic"] = t.get("dram_bytes_per_launch")
+            roofline["traffic_source"] = t.get("source")
         except Exception:
             pass
 
@@ -524,15 +557,11 @@ def main():
     torch.cuda.synchronize()
     res_host = torch.empty(LA, dtype=torch.int32, pin_memory=True)
 
+    ss_e2e = ShardedSum(ctx, LA, wl.S, wl.e2e_kernel)
+
     def e2e_step():
         wl.e2e_ingest(host)
-        wl.e2e_kernel(partial)
-        if ws > 1:
-            dist.all_gather_into_tensor(gathered, partial)
-            ctx.sum_combine(gathered, LA, out=total)
-            res_host.copy_(total, non_blocking=True)
-        else:
-            res_host.copy_(partial, non_blocking=True)
+        res_host.copy_(ss_e2e(), non_blocking=True)
 
     for _ in range(2):
         e2e_step()
@@ -553,14 +582,21 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ems = float(t.item())
     ctx.check()
-    assert up.format_decimal(res_host.tolist(), wl.S) == result, "e2e result differs from the resident run"
+    e2e_global = sum(min(E2E_MAX_ROWS, b - a) for a, b in (shard_range(n_global, ws, r) for r in range(ws)))
+    if wl.e2e_rows == rows:
+        assert up.format_decimal(res_host.tolist(), wl.S) == result, "e2e result differs from the resident run"
     h2d = sum(hb.numel() for hb in host)
-    e2e = {"value": n_global / (ems / K2 / 1e3), "unit": "tuples/s", "h2d_bytes_per_step": h2d,
+    e2e = {"value": e2e_global / (ems / K2 / 1e3), "unit": "tuples/s", "h2d_bytes_per_step": h2d,
            "d2h_bytes_per_step": LA * 4, "ms_per_step": ems / K2}
+    if wl.e2e_rows < rows:
+        e2e["rows"] = f"first {wl.e2e_rows} rows of each rank's shard ({e2e_global} in total)"
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(wl)
+        cpu, oracle_full = cpu_baseline(wl)
+        if oracle_full is not None:
+            assert oracle_full == result, f"bench SUM {result} != oracle SUM {oracle_full}"
+            cpu["parity"] = "bench result == oracle SUM over every row"
 
     if rank == 0:
         desc = {"workload": cfg["name"], "rows_per_gpu": rows, "global_rows": n_global,
@@ -571,7 +607,7 @@ def main():
         desc.update(wl.workload_desc())
         line = {
             "metric": METRIC, "value": value, "unit": "tuples/s", "n_gpus": ws, "steps": K,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": scaling,
             "vs_baseline": None, "dtype": "u32", "data": "synthetic", "config": desc,
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
             "clocks": clk.summary(), "result": result, "jit_ms": round(ctx.jit_ms, 1),

@@ -93,3 +93,74 @@ def test_gloo_two_rank_sharded_sum(n):
         assert p.exitcode == 0
     whole, got = q.get(timeout=10)
     assert got == whole
+
+
+class _OracleCtx:
+    """Test double for libup's ctx on a GPU-less host: shard SUMs by the
+    oracle, the combine by Python ints.  It lets the gloo test drive the
+    product's ShardedSum plumbing (global-N typing, host staging, all-gather
+    order, empty shards) without a GPU; the real ctx runs the same class in
+    tests/test_gpu_dist.py."""
+
+    def sum_type(self, expr, cols, n_global):
+        import oracle
+        from paper_conf_icde_lixylz24_b200 import up
+        p, s = oracle.expr_type(expr, cols)
+        P, S = oracle.sum_type(p, s, n_global)
+        return P, S, up.limbs(P)
+
+    def sum_expr(self, expr, cols, n_global, out):
+        import oracle
+        v, P, S = oracle.eval_sum(expr, cols, n_global=n_global)
+        out.copy_(torch.tensor(_to_limbs(int(v.replace(".", "")), out.numel()), dtype=torch.int32))
+        return out
+
+    def sum_combine(self, gathered, la, out):
+        tot = sum(_from_limbs(gathered[r * la:(r + 1) * la].tolist()) for r in range(gathered.numel() // la))
+        out.copy_(torch.tensor(_to_limbs(tot, la), dtype=torch.int32))
+        return out
+
+
+def _sharded_worker(rank, world, port, n, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    from gen import synth
+    from paper_conf_icde_lixylz24_b200.dist import ShardedSum
+    types = [(35, 5), (32, 2)]
+    lo, hi = shard_range(n, world, rank)
+    host = [synth.uniform_decimal(hi - lo, p, 2, k + 1, row0=lo) for k, (p, s) in enumerate(types)]
+    cols = [oracle.Column(p, s, m, g) for (m, g), (p, s) in zip(host, types)]
+    ss = ShardedSum.expr(_OracleCtx(), "c1+c2", cols, n, device=torch.device("cpu"))
+    assert ss.stage_host and ss.world == world
+    ss()
+    from paper_conf_icde_lixylz24_b200 import up
+    got = up.format_decimal([x & 0xFFFFFFFF for x in ss.result_tensor().tolist()], ss.S)
+    allg = [None] * world
+    dist.all_gather_object(allg, got)
+    assert len(set(allg)) == 1            # every rank holds the same exact total
+    if rank == 0:
+        whole_host = [synth.uniform_decimal(n, p, 2, k + 1) for k, (p, s) in enumerate(types)]
+        whole, _, _ = oracle.eval_sum("c1+c2", [oracle.Column(p, s, m, g) for (m, g), (p, s) in
+                                                zip(whole_host, types)])
+        q.put((whole, got))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,n", [(2, 1), (2, 2001), (3, 2)])
+def test_gloo_sharded_sum_plumbing(world, n):
+    """The product's ShardedSum over gloo (world 2 and 3) with a test-double
+    ctx: includes empty shards (n_global < world)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_sharded_worker, args=(r, world, port, n, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(180)
+        assert p.exitcode == 0
+    whole, got = q.get(timeout=10)
+    assert got == whole

@@ -57,6 +57,17 @@ def raw(rep):
             if key in h:
                 i = h.index(key)
                 k[key] = f"{r[i]} {units[i]}".strip()
+        # warp-stall breakdown (cycles per issued instruction, by reason)
+        stalls = {}
+        for i, key in enumerate(h):
+            if key.startswith("smsp__average_warps_issue_stalled_") and key.endswith("_per_issue_active.ratio"):
+                try:
+                    stalls[key[len("smsp__average_warps_issue_stalled_"):-len("_per_issue_active.ratio")]] = \
+                        float(r[i].replace(",", ""))
+                except ValueError:
+                    pass
+        if stalls:
+            k["stall_cycles_per_issue"] = dict(sorted(stalls.items(), key=lambda kv: -kv[1])[:12])
         res.append(k)
     return res
 
@@ -66,7 +77,8 @@ def main():
     ap.add_argument("--tag", required=True)
     ap.add_argument("--launches")
     ap.add_argument("--rep")
-    ap.add_argument("--traffic-json")
+    ap.add_argument("--traffic-json", help="write the top kernel's DRAM bytes per launch here "
+                    "(bench.py reads profiles/traffic/<workload key>.json)")
     ap.add_argument("--note", default="")
     a = ap.parse_args()
     os.makedirs("profiles", exist_ok=True)
@@ -81,6 +93,7 @@ def main():
                 v, u = f[key].split()
                 v = float(v.replace(",", ""))
                 return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[u]
+            os.makedirs(os.path.dirname(a.traffic_json) or ".", exist_ok=True)
             json.dump({"kernel": f["kernel"], "dram_bytes_per_launch": mb("dram__bytes_read.sum") + mb("dram__bytes_write.sum"),
                        "source": a.rep, "tag": a.tag}, open(a.traffic_json, "w"), indent=1)
     json.dump(summ, open(f"profiles/{a.tag}.json", "w"), indent=1)
