@@ -152,11 +152,14 @@ class ExprWorkload(Workload):
             mag, neg = gdev.uniform_decimal(self.rows, p, self.args.config, k + 1, row0=self.row0,
                                             nonzero_lead=(k in cfg.get("lead", ())))
             self.raw.append((mag, neg))
-            self.cols.append(ctx.column_from_device_bin(p, s, mag, neg))
+            self.cols.append(ctx.column_from_device_bin(p, s, mag, neg, layout=self.args.layout))
         ctx.check()
         self.P, self.S, self.LA = ctx.sum_type(cfg["expr"], self.cols, self.n_global)
-        self.e2e_cols = [up.Column(p, s, self.e2e_rows) for p, s in cfg["types"]]
-        self.bytes_per_row = sum(4 * up.limbs(p) for p, s in cfg["types"])
+        self.e2e_cols = [up.Column(p, s, self.e2e_rows, layout=self.args.layout) for p, s in cfg["types"]]
+        # algorithmic bytes per row: the columns as stored -- limb planes (4 B per
+        # limb) or the paper's compact rows (Lb bytes)
+        self.bytes_per_row = sum((up.compact_bytes(p) if self.args.layout == "compact" else 4 * up.limbs(p))
+                                 for p, s in cfg["types"])
 
     def kernel(self, out):
         self.ctx.sum_expr(self.cfg["expr"], self.cols, self.n_global, out=out)
@@ -178,6 +181,8 @@ class ExprWorkload(Workload):
 
     def e2e_ingest(self, host):
         for hb, (p, s), col in zip(host, self.cfg["types"], self.e2e_cols):
+            # compact layout: the host rows land in place (H2D + range check);
+            # planes: H2D + in-kernel expand into limb planes
             self.ctx.column_from_compact(p, s, hb, n=self.e2e_rows, out=col)
 
     def e2e_kernel(self, out):
@@ -197,7 +202,8 @@ class ExprWorkload(Workload):
         ach = alg / (kernel_ms / 1e3) / 1e9
         r = {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
              "frac": round(ach / peak, 4), "kernel_ms": round(kernel_ms, 5), "alg_bytes_per_launch": alg,
-             "alg_unit": f"{self.bytes_per_row} B/row (limb planes of all columns) x {self.rows} rows",
+             "alg_unit": f"{self.bytes_per_row} B/row ({'compact rows' if self.args.layout == 'compact' else 'limb planes'}"
+                         f" of all columns) x {self.rows} rows",
              "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks
              else "fallback 6.65 TB/s"}
         if self.cfg["types"][0][0] >= 100:
@@ -421,6 +427,8 @@ def main():
     ap.add_argument("--rows", type=int, default=0, help="rows per GPU (default: the config's)")
     ap.add_argument("--global-rows", type=int, default=0, help="total rows, sharded over the GPUs (strong scaling)")
     ap.add_argument("--impl", default="up", choices=["up", "reference"])
+    ap.add_argument("--layout", default="planes", choices=["planes", "compact"],
+                    help="column storage for the expression configs (1-3): limb planes or the paper's compact rows")
     ap.add_argument("--ref-rows", type=int, default=200_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=0)
@@ -605,6 +613,8 @@ def main():
                 "l2": ("flushed before every step (256 MB write, then a 256 MB read that writes the dirty lines back)" if flush is not None
                        else "inputs larger than L2 or compute-bound (no flush)")}
         desc.update(wl.workload_desc())
+        if cfg["kind"] == "expr":
+            desc["layout"] = args.layout
         line = {
             "metric": METRIC, "value": value, "unit": "tuples/s", "n_gpus": ws, "steps": K,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": scaling,

@@ -62,9 +62,25 @@ up_status up_ctx_destroy(up_ctx *ctx);
  */
 typedef struct {
     int64_t n, ld;
-    int32_t p, s, limbs, reserved;
+    int32_t p, s, limbs, layout;
     uint32_t *data;
 } up_column;
+
+/*
+ * Column layouts (up_column.layout):
+ *  UP_LAYOUT_PLANES  -- limb planes as above (every entry point).
+ *  UP_LAYOUT_COMPACT -- the paper's compact byte rows (cDecimal, P:L843-873,
+ *     Fig. 4) kept resident on the device: row i is the Lb = up_compact_bytes(p)
+ *     bytes at ((uint8_t *)data)[i*Lb], little-endian magnitude, sign in the
+ *     top bit of the last byte; ld must equal Lb; data 16-byte aligned and the
+ *     allocation at least n*Lb rounded up to 16 bytes (kernels read whole
+ *     16-byte vectors).  Read directly (no limb planes materialised) by
+ *     up_eval_expr / up_sum_expr / up_sum / up_filter inputs;
+ *     ingestion: up_column_from_{host,device}_compact copy the rows in place
+ *     (+ range check), the _bin / string calls convert.  Other entry points
+ *     return UP_E_UNSUPPORTED for compact inputs.
+ */
+enum { UP_LAYOUT_PLANES = 0, UP_LAYOUT_COMPACT = 1 };
 
 /* Limb count L = min{L : 10^p <= 2^(32L-1)} (reading Q1 of P:L821-837 vs
  * reproduces 18/38/76/153/307 <-> 2/4/8/16/32). */

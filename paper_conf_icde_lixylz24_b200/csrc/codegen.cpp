@@ -238,13 +238,16 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     const bool narrow = max_limbs(root) <= 8 && !uses_divmod(root);
     const int R = narrow ? 4 : 1;
     info.rows_per_thread = R;
+    bool any_compact = false;
+    for (size_t c = 0; c < cols.size(); ++c) any_compact = any_compact || (used[c] && cols[c].Lb > 0);
 
     Emitter E;
     {
         std::vector<int> uses(cols.size(), 0), div_uses(cols.size(), 0);
         div_only_uses(root, uses, div_uses);
         E.lazy.assign(cols.size(), false);
-        for (size_t c = 0; c < cols.size(); ++c) E.lazy[c] = used[c] && uses[c] > 0 && uses[c] == div_uses[c];
+        for (size_t c = 0; c < cols.size(); ++c)
+            E.lazy[c] = used[c] && cols[c].Lb == 0 && uses[c] > 0 && uses[c] == div_uses[c];
     }
     std::string res = E.emit(root);
 
@@ -292,10 +295,69 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
         else k << "    AccChain<" << LOUT << "," << KC << "> acc; acc.init();\n";
     }
     k << "    const long long n = P.n;\n";
-    k << "    const long long stride = (long long)gridDim.x * blockDim.x * R;\n";
-    k << "    for (long long base = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * R; base < n; base += stride) {\n";
+    if (any_compact) {
+        // Compact columns (NEXT-2, the paper's cDecimal rows read in place,
+        // P:L843-873, Listing 1's expand step P:L942-948): per block tile of
+        // 256 R rows, each compact column's tile bytes (256 R Lb, a multiple
+        // of 16) arrive in shared memory with coalesced 16-byte streaming loads;
+        // each thread then assembles its R rows' two's-complement limbs there.
+        for (size_t c = 0; c < cols.size(); ++c) {
+            if (!used[c] || cols[c].Lb == 0) continue;
+            k << "    __shared__ __align__(16) u32 cs" << c << "[" << (256 * R * cols[c].Lb) / 4 + 4 << "];\n";
+        }
+        k << "    constexpr long long TILE = 256 * R;\n";
+        k << "    for (long long t0 = (long long)blockIdx.x * TILE; t0 < n; t0 += (long long)gridDim.x * TILE) {\n";
+        for (size_t c = 0; c < cols.size(); ++c) {
+            if (!used[c] || cols[c].Lb == 0) continue;
+            const int Lb = cols[c].Lb;
+            k << "        { const uint4 *src = reinterpret_cast<const uint4 *>(reinterpret_cast<const unsigned char *>(P.col[" << c
+              << "]) + t0 * " << Lb << ");\n";
+            k << "          const int nv = (int)(((n - t0 < TILE ? n - t0 : TILE) * " << Lb << " + 15) / 16);\n";
+            k << "          for (int i = threadIdx.x; i < nv; i += 256) reinterpret_cast<uint4 *>(cs" << c << ")[i] = __ldcs(src + i); }\n";
+        }
+        k << "        __syncthreads();\n";
+        k << "        const long long base = t0 + (long long)threadIdx.x * R;\n";
+    } else {
+        k << "    const long long stride = (long long)gridDim.x * blockDim.x * R;\n";
+        k << "    for (long long base = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * R; base < n; base += stride) {\n";
+    }
     for (size_t c = 0; c < cols.size(); ++c) {
-        if (!used[c] || E.lazy[c]) continue;
+        if (!used[c] || cols[c].Lb == 0) continue;
+        // thread's rows: tile bytes [tid R Lb, (tid + 1) R Lb); row r's limbs by
+        // funnel shifts, the sign = top bit of its last byte, then two's complement
+        const int Lc = cols[c].limbs, Lb = cols[c].Lb;
+        const int NW = (R * Lb + 3) / 4 + 1;
+        k << "        u32 x" << c << "[R][" << Lc << "];\n";
+        k << "        { const int b0 = (int)threadIdx.x * " << R * Lb << ";\n";
+        k << "          const u32 *w = cs" << c << " + (b0 >> 2); const u32 sh0 = (u32)(b0 & 3) * 8u;\n";
+        k << "          u32 wv[" << NW + 1 << "];\n";
+        k << "#pragma unroll\n          for (int i = 0; i < " << NW + 1 << "; ++i) wv[i] = w[i];\n";
+        k << "          u32 al[" << NW << "];   // the thread's bytes, word-aligned\n";
+        k << "#pragma unroll\n          for (int i = 0; i < " << NW << "; ++i) al[i] = __funnelshift_r(wv[i], wv[i + 1], sh0);\n";
+        for (int r = 0; r < R; ++r) {
+            const int rb = r * Lb;                      // row byte offset in al[]
+            const int sbit = 8 * (rb + Lb - 1) + 7;    // sign bit (absolute bit in al[])
+            k << "          { const u32 ng = (al[" << sbit / 32 << "] >> " << sbit % 32 << ") & 1u; const u32 m = 0u - ng; u64 cy = ng;\n";
+            for (int j = 0; j < Lc; ++j) {
+                const int bit0 = 8 * rb + 32 * j;       // limb j's first bit in al[]
+                const int mag_bits = 8 * Lb - 1 - 32 * j;   // magnitude bits left in this row from limb j
+                std::string v;
+                if (mag_bits <= 0) v = "0u";
+                else {
+                    v = (bit0 % 32) ? "__funnelshift_r(al[" + std::to_string(bit0 / 32) + "], al[" + std::to_string(bit0 / 32 + 1) +
+                                          "], " + std::to_string(bit0 % 32) + "u)"
+                                    : "al[" + std::to_string(bit0 / 32) + "]";
+                    if (mag_bits < 32) v = "(" + v + " & " + std::to_string((1u << mag_bits) - 1u) + "u)";
+                }
+                k << "            { const u64 t = (u64)(" << v << " ^ m) + cy; x" << c << "[" << r << "][" << j
+                  << "] = (u32)t; cy = t >> 32; }\n";
+            }
+            k << "          }\n";
+        }
+        k << "        }\n";
+    }
+    for (size_t c = 0; c < cols.size(); ++c) {
+        if (!used[c] || E.lazy[c] || cols[c].Lb > 0) continue;
         const int Lc = cols[c].limbs;
         k << "        u32 x" << c << "[R][" << Lc << "];\n";
         k << "        { const u32 *p = P.col[" << c << "] + base; const long long ld = P.ld[" << c << "];\n";
@@ -335,6 +397,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
         else
             k << "#pragma unroll\n        for (int j = 0; j < " << LOUT << "; ++j) __stcs(P.out + j * P.ld_out + base, res[0][j]);\n";
     }
+    if (any_compact) k << "        __syncthreads();\n";
     k << "    }\n";
     k << "    if (fl) atomicOr(P.flags, fl);\n";
     if (opt.sum) {

@@ -19,7 +19,9 @@ struct Node {
     std::unique_ptr<Node> l, r;
 };
 
-struct ColType { int p, s, limbs; };
+// Lb > 0: the column is stored in the compact byte layout (the paper's
+// cDecimal): Lb bytes per row, row-major; else limb planes
+struct ColType { int p, s, limbs; int Lb = 0; };
 
 // Parse "c1*c2 - c3/c4" (SQL precedence, left-assoc, unary -, parentheses,
 // literals typed by value: 1.23 -> DECIMAL(3,2), 10 -> DECIMAL(2,0),

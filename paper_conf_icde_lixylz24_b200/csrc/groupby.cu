@@ -96,6 +96,7 @@ extern "C" up_status up_group_ids(up_ctx *c, const up_column *keys, int nkeys, i
     for (int k = 0; k < nkeys; ++k) {
         const up_column &col = keys[k];
         if (col.n != n) return up_internal_fail(UP_E_INVAL, "group_ids: key columns differ in length");
+        if (col.layout != UP_LAYOUT_PLANES) return up_internal_fail(UP_E_UNSUPPORTED, "group_ids: key columns must be limb planes");
         if (col.p < 1 || col.limbs != up_limbs(col.p) || (n > 0 && !col.data) || col.ld < n)
             return up_internal_fail(UP_E_INVAL, "group_ids: bad key column descriptor");
         for (int j = 0; j < col.limbs; ++j) {

@@ -154,7 +154,7 @@ __global__ void __launch_bounds__(256) k_from_compact(const uint8_t *__restrict_
             if (cmp >= 0) fl |= up::F_RANGE;
             u64 carry = ng;
             const long long i = base + threadIdx.x;
-            for (int j = 0; j < L; ++j) {
+            for (int j = 0; out && j < L; ++j) {   // out == nullptr: range check only (compact-resident column)
                 u32 m = 0;
                 for (int b = 0; b < 4; ++b) {
                     const int k = 4 * j + b;

@@ -207,12 +207,16 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
             const u64 smsk = negt ? ~0ull : 0ull;
 #endif
             const u32 nd1 = 0u - d1;
+            // software pipeline: the digit step tau + 1 consumes was written at step <= tau - 1
+            // (DELTA >= 6 + sd), so it is loaded one step ahead, off the remainder chain
+            u32 ynext = lds32p((unsigned)jb <= (unsigned)jtop && jb >= jld, yl);
 #pragma unroll 2
             for (int tau = 0; tau < steps; ++tau) {
                 const int j = jb - tau;
                 const bool act = (unsigned)j <= (unsigned)jtop;
                 const bool ld = act && j >= jld;
-                const u32 y = lds32p(ld, yl);
+                const u32 y = ynext;
+                ynext = lds32p((unsigned)(j - 1) <= (unsigned)jtop && j - 1 >= jld, yl - 4u * RSY);
                 {   // running sum: S 2^c += (-1)^(k-1) Y_k 2^(c - o_k)   (y = 0: no-op)
 #if NEGSH0
                     const u64 a = ((u64)y << esh) ^ xm;
@@ -386,7 +390,7 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
         tab.insert(tab.end(), {(uint32_t)dn, (uint32_t)(dn >> 32), (uint32_t)v, (uint32_t)sh});
         sdmax = std::max(sdmax, sh >> 5);
     }
-    const int DELTA = 5 + sdmax;
+    const int DELTA = 6 + sdmax;   // load one step ahead + the one-step carry fix-up window
     const int WY = W + G + 8 + sdmax;
     const int WS = WY + 2;
     // S scale c = max o_k, single-slot adds when sum_rows(addends) stays < 2^62

@@ -204,9 +204,26 @@ up_status check_column(const up_column *col, const char *what) {
     if (col->p < 1 || col->s < 0) return fail(UP_E_INVAL, "%s: bad DECIMAL(%d,%d)", what, col->p, col->s);
     if (col->limbs != limbs_for_precision(col->p))
         return fail(UP_E_INVAL, "%s: limbs %d != up_limbs(%d) = %d", what, col->limbs, col->p, limbs_for_precision(col->p));
+    if (col->layout != UP_LAYOUT_PLANES && col->layout != UP_LAYOUT_COMPACT)
+        return fail(UP_E_INVAL, "%s: unknown layout %d", what, col->layout);
+    if (col->layout == UP_LAYOUT_COMPACT) {
+        if (col->ld != up_compact_bytes(col->p))
+            return fail(UP_E_INVAL, "%s: compact column needs ld = up_compact_bytes(%d) = %d", what, col->p, up_compact_bytes(col->p));
+        if (col->n < 0) return fail(UP_E_INVAL, "%s: bad n", what);
+        if (col->n > 0 && (!col->data || ((uintptr_t)col->data & 15))) return fail(UP_E_INVAL, "%s: data must be 16-byte aligned device memory", what);
+        if (col->n >= (1ll << 32)) return fail(UP_E_UNSUPPORTED, "%s: more than 2^32-1 rows per call", what);
+        return UP_OK;
+    }
     if (col->n < 0 || col->ld < col->n || (col->ld & 3)) return fail(UP_E_INVAL, "%s: bad n/ld (%lld/%lld)", what, (long long)col->n, (long long)col->ld);
     if (col->n > 0 && (!col->data || ((uintptr_t)col->data & 15))) return fail(UP_E_INVAL, "%s: data must be 16-byte aligned device memory", what);
     if (col->n >= (1ll << 32)) return fail(UP_E_UNSUPPORTED, "%s: more than 2^32-1 rows per call", what);
+    return UP_OK;
+}
+
+up_status need_planes(const up_column *col, const char *what) {
+    if (col && col->layout == UP_LAYOUT_COMPACT)
+        return fail(UP_E_UNSUPPORTED, "%s: this call needs a limb-plane column (compact columns: up_eval_expr / "
+                                      "up_sum_expr / up_filter)", what);
     return UP_OK;
 }
 
@@ -320,7 +337,8 @@ up_status type_expr(const char *expr, const up_column *cols, int ncols, Typed &t
     for (int i = 0; i < ncols; ++i) {
         if (cols[i].p < 1 || cols[i].s < 0 || cols[i].limbs != limbs_for_precision(cols[i].p))
             return fail(UP_E_INVAL, "column %d: bad type/limbs", i + 1);
-        t.types.push_back({cols[i].p, cols[i].s, cols[i].limbs});
+        t.types.push_back({cols[i].p, cols[i].s, cols[i].limbs,
+                           cols[i].layout == UP_LAYOUT_COMPACT ? up_compact_bytes(cols[i].p) : 0});
     }
     std::string err;
     t.root = parse_expr(expr, ncols, err);
@@ -333,7 +351,8 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     std::string k = tag;
     k += '|';
     k += expr;
-    for (int i = 0; i < ncols; ++i) k += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
+    for (int i = 0; i < ncols; ++i)
+        k += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s) + (cols[i].layout == UP_LAYOUT_COMPACT ? "c" : "");
     k += "|" + std::to_string(extra);
     if (getenv("UP_NO_OPT")) k += "|noopt";
     if (getenv("UP_NO_WIDE")) k += "|nowide";
@@ -375,7 +394,9 @@ up_status expr_kernel(up_ctx *c, const char *expr, const up_column *cols, int nc
     std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(t.root.get(), t.types);
     const Node *gen_root = opt_root ? opt_root.get() : t.root.get();
     // wide SUM regime: warp per row, linear decomposition into summed terms
-    if (sum && max_limbs(gen_root) >= kWideMinLimbs && LA <= 512 && !getenv("UP_NO_WIDE"))
+    bool any_compact = false;
+    for (const ColType &ct : t.types) any_compact = any_compact || ct.Lb > 0;
+    if (sum && !any_compact && max_limbs(gen_root) >= kWideMinLimbs && LA <= 512 && !getenv("UP_NO_WIDE"))
         src = gen_wide_sum_kernel(gen_root, t.types, LA, info);
     if (src.empty()) {
         info = GenInfo();
@@ -441,6 +462,8 @@ void fill_cols(up_kparams &P, const up_column *cols, int ncols) {
 
 }  // namespace
 
+up_status scratch_locked(up_ctx *c, size_t bytes, void **out);   // ctx scratch; caller holds c->mu
+
 // ====================================================================== C ABI
 extern "C" {
 
@@ -501,6 +524,15 @@ up_status up_column_from_device_bin(up_ctx *c, const uint32_t *d_mag, int32_t W,
     std::lock_guard<std::mutex> g(c->mu);
     const uint32_t *bound = nullptr;
     if (up_status s = pow10_device(c, dst->p, &bound)) return s;
+    if (dst->layout == UP_LAYOUT_COMPACT) {   // via limb planes in the ctx scratch
+        const long long ld = (dst->n + 3) & ~3ll;
+        uint32_t *planes = nullptr;
+        if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)dst->limbs * (size_t)ld, (void **)&planes)) return s;
+        CUDA_TRY(upk_launch_from_bin(d_mag, W, d_neg, dst->n, bound, dst->limbs, planes, ld, c->d_flags, (cudaStream_t)stream));
+        CUDA_TRY(upk_launch_to_compact(planes, dst->limbs, ld, dst->n, (uint8_t *)dst->data, (int)dst->ld, (cudaStream_t)stream));
+        c->launches += 2;
+        return UP_OK;
+    }
     CUDA_TRY(upk_launch_from_bin(d_mag, W, d_neg, dst->n, bound, dst->limbs, dst->data, dst->ld, c->d_flags,
                                  (cudaStream_t)stream));
     c->launches++;
@@ -578,6 +610,15 @@ up_status up_column_from_device_compact(up_ctx *c, const uint8_t *d_bytes, up_co
     std::lock_guard<std::mutex> g(c->mu);
     const uint32_t *bound = nullptr;
     if (up_status s = pow10_device(c, dst->p, &bound)) return s;
+    if (dst->layout == UP_LAYOUT_COMPACT) {   // stays compact: copy + range check (no planes written)
+        const size_t nb = (size_t)dst->ld * (size_t)dst->n;
+        if ((const void *)d_bytes != (const void *)dst->data)
+            CUDA_TRY(cudaMemcpyAsync(dst->data, d_bytes, nb, cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+        CUDA_TRY(upk_launch_from_compact((const uint8_t *)dst->data, (int)dst->ld, dst->n, bound, dst->limbs, nullptr, 0,
+                                         c->d_flags, (cudaStream_t)stream));
+        c->launches++;
+        return UP_OK;
+    }
     CUDA_TRY(upk_launch_from_compact(d_bytes, up_compact_bytes(dst->p), dst->n, bound, dst->limbs, dst->data, dst->ld,
                                      c->d_flags, (cudaStream_t)stream));
     c->launches++;
@@ -590,6 +631,12 @@ up_status up_column_from_host_compact(up_ctx *c, const uint8_t *bytes, up_column
     if (dst->n == 0) return UP_OK;
     cudaStream_t st = (cudaStream_t)stream;
     const size_t nb = (size_t)up_compact_bytes(dst->p) * (size_t)dst->n;
+    if (dst->layout == UP_LAYOUT_COMPACT) {   // rows land in place: H2D + range check, no conversion
+        CUDA_TRY(cudaMemcpyAsync(dst->data, bytes, nb, cudaMemcpyHostToDevice, st));
+        if (up_status s = up_column_from_device_compact(c, (const uint8_t *)dst->data, dst, stream)) return s;
+        CUDA_TRY(cudaStreamSynchronize(st));   // up.h: host buffer reusable on return
+        return UP_OK;
+    }
     {
         std::lock_guard<std::mutex> g(c->mu);
         if (up_status s = ensure_stage(c, nb, st)) return s;
@@ -607,6 +654,11 @@ up_status up_column_to_host_compact(up_ctx *c, const up_column *col, uint8_t *by
     cudaStream_t st = (cudaStream_t)stream;
     const int Lb = up_compact_bytes(col->p);
     const size_t nb = (size_t)Lb * (size_t)col->n;
+    if (col->layout == UP_LAYOUT_COMPACT) {
+        CUDA_TRY(cudaMemcpyAsync(bytes, col->data, nb, cudaMemcpyDeviceToHost, st));
+        CUDA_TRY(cudaStreamSynchronize(st));
+        return UP_OK;
+    }
     std::lock_guard<std::mutex> g(c->mu);
     if (up_status s = ensure_stage(c, nb, st)) return s;
     CUDA_TRY(upk_launch_to_compact(col->data, col->limbs, col->ld, col->n, (uint8_t *)c->d_stage, Lb, st));
@@ -627,7 +679,20 @@ up_status up_column_to_host_bin(up_ctx *c, const up_column *col, uint32_t *mag, 
     if (up_status s = ensure_stage(c, mb_al + nb, st)) return s;
     uint32_t *dm = (uint32_t *)c->d_stage;
     uint8_t *dn = (uint8_t *)c->d_stage + mb_al;
-    CUDA_TRY(upk_launch_to_bin(col->data, col->limbs, col->ld, col->n, dm, dn, st));
+    const uint32_t *planes = col->data;
+    long long ld = col->ld;
+    if (col->layout == UP_LAYOUT_COMPACT) {   // compact -> limb planes in the ctx scratch first
+        ld = (col->n + 3) & ~3ll;
+        uint32_t *pl = nullptr;
+        if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)col->limbs * (size_t)ld, (void **)&pl)) return s;
+        const uint32_t *bound = nullptr;
+        if (up_status s = pow10_device(c, col->p, &bound)) return s;
+        CUDA_TRY(upk_launch_from_compact((const uint8_t *)col->data, (int)col->ld, col->n, bound, col->limbs, pl, ld,
+                                         c->d_flags, st));
+        c->launches++;
+        planes = pl;
+    }
+    CUDA_TRY(upk_launch_to_bin(planes, col->limbs, ld, col->n, dm, dn, st));
     c->launches++;
     CUDA_TRY(cudaMemcpyAsync(mag, dm, mb, cudaMemcpyDeviceToHost, st));
     CUDA_TRY(cudaMemcpyAsync(neg, dn, nb, cudaMemcpyDeviceToHost, st));
@@ -747,7 +812,10 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     // (TMA row coordinates are 32-bit signed: more rows per call take the CUDA-core contraction)
     const bool use_tc = getenv("UP_NO_TC") == nullptr && cols[0].n < (1ll << 31);
     bool try_split = getenv("UP_SPLIT") != nullptr;
-    if (!try_split && !getenv("UP_NO_SPLIT")) {
+    bool any_compact = false;
+    for (int i = 0; i < ncols; ++i) any_compact = any_compact || cols[i].layout == UP_LAYOUT_COMPACT;
+    if (any_compact) try_split = false;   // the row contractions read limb planes (TMA boxes)
+    else if (!try_split && !getenv("UP_NO_SPLIT")) {
         const long thr = use_tc ? kContractMinProducts : kSplitAutoProducts;
         for (int i = 0; i < ncols && !try_split; ++i)
             for (int j = 0; j < ncols && !try_split; ++j)
@@ -1028,6 +1096,7 @@ up_status up_group_aggregate(up_ctx *c, int32_t n_aggs, const int32_t *kinds, co
     if (!c || !cols || ncols < 1 || !d_out || !d_counts) return fail(UP_E_INVAL, "need a ctx, columns, d_out and d_counts");
     for (int i = 0; i < ncols; ++i) {
         if (up_status s = check_column(&cols[i], "input")) return s;
+        if (up_status s = need_planes(&cols[i], "group_aggregate input")) return s;
         if (cols[i].n != cols[0].n) return fail(UP_E_INVAL, "columns differ in length");
     }
     if (!d_group && n_groups != 1) return fail(UP_E_INVAL, "d_group == NULL needs n_groups == 1");
@@ -1198,6 +1267,8 @@ unsigned long long *up_internal_ws(up_ctx *c) { return c->d_ws; }
 uint32_t *up_internal_ticket(up_ctx *c) { return c->d_ticket; }
 uint32_t *up_internal_flags(up_ctx *c) { return c->d_flags; }
 int up_internal_num_sms(up_ctx *c) { return c->num_sms; }
+up_status up_internal_scratch(up_ctx *c, size_t bytes, void **out);
+up_status scratch_locked(up_ctx *c, size_t bytes, void **out) { return up_internal_scratch(c, bytes, out); }
 up_status up_internal_scratch(up_ctx *c, size_t bytes, void **out) {
     if (bytes > c->scratch_bytes) {
         if (c->d_scratch) {

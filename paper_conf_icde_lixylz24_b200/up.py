@@ -27,7 +27,7 @@ class UpError(RuntimeError):
 
 class up_column(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("ld", ctypes.c_int64), ("p", ctypes.c_int32),
-                ("s", ctypes.c_int32), ("limbs", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("s", ctypes.c_int32), ("limbs", ctypes.c_int32), ("layout", ctypes.c_int32),
                 ("data", ctypes.c_void_p)]
 
 
@@ -135,21 +135,32 @@ def _stream_ptr(stream) -> Optional[int]:
     return stream.cuda_stream
 
 
-class Column:
-    """A DECIMAL(p,s) column on the GPU: `limbs` two's-complement limb planes
-    held in a torch int32 tensor of shape (limbs, ld)."""
+LAYOUT_PLANES, LAYOUT_COMPACT = 0, 1
 
-    def __init__(self, p: int, s: int, n: int, device="cuda", data=None):
+
+class Column:
+    """A DECIMAL(p,s) column on the GPU.  layout "planes": `limbs`
+    two's-complement limb planes in a torch int32 tensor (limbs, ld);
+    layout "compact": the paper's compact byte rows (Lb = compact_bytes(p)
+    bytes per row, up.h UP_LAYOUT_COMPACT) in a uint8 tensor padded to 16 bytes."""
+
+    def __init__(self, p: int, s: int, n: int, device="cuda", data=None, layout: str = "planes"):
         import torch
         self.p, self.s, self.n = p, s, n
         self.limbs = limbs(p)
-        self.ld = ld_for(n)
-        if data is None:
-            data = torch.empty((self.limbs, max(self.ld, 4)), dtype=torch.int32, device=device)
+        self.layout = LAYOUT_COMPACT if layout == "compact" else LAYOUT_PLANES
+        if self.layout == LAYOUT_COMPACT:
+            self.ld = compact_bytes(p)
+            if data is None:
+                data = torch.empty(((n * self.ld + 15) // 16) * 16 + 16, dtype=torch.uint8, device=device)
+        else:
+            self.ld = ld_for(n)
+            if data is None:
+                data = torch.empty((self.limbs, max(self.ld, 4)), dtype=torch.int32, device=device)
         self.data = data
 
     def desc(self) -> up_column:
-        return up_column(self.n, self.ld, self.p, self.s, self.limbs, 0, self.data.data_ptr())
+        return up_column(self.n, self.ld, self.p, self.s, self.limbs, self.layout, self.data.data_ptr())
 
     @property
     def type(self):
@@ -215,7 +226,8 @@ class Context:
         return lib().up_jit_ms(self.h)
 
     # ------------------------------------------------------------------ columns
-    def column_from_host_bin(self, p: int, s: int, mag, neg=None, stream=None, out: Optional[Column] = None):
+    def column_from_host_bin(self, p: int, s: int, mag, neg=None, stream=None, out: Optional[Column] = None,
+                             layout: str = "planes"):
         """mag: (n, W) uint32 host array (numpy or pinned torch); neg: (n,) uint8."""
         import numpy as np
         import torch
@@ -227,15 +239,16 @@ class Context:
             n, W = mag.shape
             mag_ptr = mag.data_ptr()
             neg_ptr = neg.data_ptr() if neg is not None else None
-        col = out if out is not None else Column(p, s, n)
+        col = out if out is not None else Column(p, s, n, layout=layout)
         d = col.desc()
         _chk(lib().up_column_from_host_bin(self.h, mag_ptr, W, neg_ptr, ctypes.byref(d), _stream_ptr(stream)))
         return col
 
-    def column_from_device_bin(self, p: int, s: int, d_mag, d_neg=None, stream=None, out: Optional[Column] = None):
+    def column_from_device_bin(self, p: int, s: int, d_mag, d_neg=None, stream=None, out: Optional[Column] = None,
+                               layout: str = "planes"):
         """d_mag: (n, W) int32/uint32 CUDA tensor; d_neg: (n,) uint8 CUDA tensor."""
         n, W = d_mag.shape
-        col = out if out is not None else Column(p, s, n)
+        col = out if out is not None else Column(p, s, n, layout=layout)
         d = col.desc()
         _chk(lib().up_column_from_device_bin(self.h, d_mag.data_ptr(), W,
                                              d_neg.data_ptr() if d_neg is not None else None,
@@ -243,7 +256,7 @@ class Context:
         return col
 
     def column_from_compact(self, p: int, s: int, data, n: Optional[int] = None, stream=None,
-                            out: Optional[Column] = None):
+                            out: Optional[Column] = None, layout: str = "planes"):
         """Compact rows: numpy uint8 / pinned torch uint8 (host) or a CUDA uint8 tensor."""
         import numpy as np
         Lb = compact_bytes(p)
@@ -253,7 +266,7 @@ class Context:
         else:
             n = data.numel() // Lb if n is None else n
             ptr, dev = data.data_ptr(), data.is_cuda
-        col = out if out is not None else Column(p, s, n)
+        col = out if out is not None else Column(p, s, n, layout=layout)
         d = col.desc()
         fn = lib().up_column_from_device_compact if dev else lib().up_column_from_host_compact
         _chk(fn(self.h, ptr, ctypes.byref(d), _stream_ptr(stream)))
@@ -266,8 +279,8 @@ class Context:
         _chk(lib().up_column_to_host_compact(self.h, ctypes.byref(d), out.ctypes.data, _stream_ptr(stream)))
         return out[: col.n * compact_bytes(col.p)]
 
-    def column_from_strings(self, p: int, s: int, values: Sequence[str], stream=None):
-        col = Column(p, s, len(values))
+    def column_from_strings(self, p: int, s: int, values: Sequence[str], stream=None, layout: str = "planes"):
+        col = Column(p, s, len(values), layout=layout)
         arr = (ctypes.c_char_p * max(1, len(values)))(*[v.encode() for v in values])
         d = col.desc()
         _chk(lib().up_column_from_host(self.h, arr, ctypes.byref(d), _stream_ptr(stream)))
@@ -485,10 +498,15 @@ def result_to_string(limb_tensor, s: int) -> str:
 
 
 # ---------------------------------------------------------------------- diagnostics
-def gen_source(variant: str, expr: str, types: Sequence[tuple], n_global: int = 1) -> str:
+def gen_source(variant: str, expr: str, types: Sequence[tuple], n_global: int = 1,
+               compact: Optional[Sequence[bool]] = None) -> str:
+    """Generated kernel source (no GPU); compact[i]: column i in the compact layout."""
     arr = (up_column * max(1, len(types)))()
     for i, (p, s) in enumerate(types):
-        arr[i] = up_column(n_global, ld_for(n_global), p, s, limbs(p), 0, None)
+        if compact and compact[i]:
+            arr[i] = up_column(n_global, compact_bytes(p), p, s, limbs(p), LAYOUT_COMPACT, None)
+        else:
+            arr[i] = up_column(n_global, ld_for(n_global), p, s, limbs(p), 0, None)
     buf = ctypes.create_string_buffer(1 << 24)
     _chk(lib().up_gen_source(variant.encode(), expr.encode(), arr, len(types), n_global, buf, len(buf)))
     return buf.value.decode()
