@@ -183,8 +183,8 @@ up_status up_sum_combine(up_ctx *ctx, const uint32_t *d_partials, int32_t nranks
  *   total sum_a n_groups * limbs_a uint32.
  * d_counts (device): n_groups uint64 row counts (COUNT(*) per group).  An
  *   empty group yields 0 for every aggregate (SQL NULL; see its count).
- * Errors raised by rows of excluded groups are not flagged.  Single-GPU
- * (MIN/MAX/AVG partials do not combine by up_sum_combine).
+ * Errors raised by rows of excluded groups are not flagged.  Across ranks:
+ * up_group_combine below.
  */
 typedef enum { UP_AGG_SUM = 0, UP_AGG_MIN = 1, UP_AGG_MAX = 2, UP_AGG_AVG = 3 } up_agg_kind;
 up_status up_agg_type(const char *expr, int32_t kind, const up_column *cols, int ncols, int64_t n_global,
@@ -192,6 +192,24 @@ up_status up_agg_type(const char *expr, int32_t kind, const up_column *cols, int
 up_status up_group_aggregate(up_ctx *ctx, int32_t n_aggs, const int32_t *kinds, const char *const *exprs,
                              const up_column *cols, int ncols, const int32_t *d_group, int32_t n_groups,
                              int64_t n_global, uint32_t *d_out, uint64_t *d_counts, void *stream);
+
+/*
+ * Multi-rank GROUP BY (NEXT-4 with rows a13/e): every rank runs
+ * up_group_aggregate over its rows with each AVG replaced by SUM (the
+ * combinable partial state of an average; same n_global on every rank), the
+ * packed outputs and the counts are all-gathered rank-major (d_parts:
+ * nranks x that layout's words, d_counts: nranks x n_groups uint64), then
+ * this call writes the final results in up_group_aggregate's layout for the
+ * ORIGINAL kinds: SUM = exact sum over ranks; MIN / MAX over the ranks whose
+ * group is non-empty; AVG = trunc(|SUM| 10^4 / COUNT) sign(SUM) of the
+ * combined SUM and COUNT (reading Q4; COUNT 0 -> 0).
+ * d_counts_out (optional): n_groups combined counts.  One kernel launch;
+ * aggregates wider than 80 limbs: UP_E_UNSUPPORTED.
+ */
+up_status up_group_combine(up_ctx *ctx, int32_t n_aggs, const int32_t *kinds, const char *const *exprs,
+                           const up_column *cols, int ncols, int32_t n_groups, int64_t n_global,
+                           const uint32_t *d_parts, int32_t nranks, const uint64_t *d_counts, uint32_t *d_out,
+                           uint64_t *d_counts_out, void *stream);
 
 /*
  * WHERE lhs <op> rhs (the DECIMAL comparison

@@ -297,29 +297,55 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     k << "    const long long n = P.n;\n";
     if (any_compact) {
         // Compact columns (NEXT-2, the paper's cDecimal rows read in place,
-        // P:L843-873, Listing 1's expand step P:L942-948): per block tile of
-        // 256 R rows, each compact column's tile bytes (256 R Lb, a multiple
-        // of 16) arrive in shared memory with coalesced 16-byte streaming loads;
-        // each thread then assembles its R rows' two's-complement limbs there.
+        // P:L843-873, Listing 1's expand step P:L942-948): tiles of 256 R rows;
+        // each compact column's tile bytes (256 R Lb, a multiple of 16) are
+        // brought into shared memory by ONE 1-D TMA bulk copy (cp.async.bulk)
+        // completing on an mbarrier, double-buffered: the copy of the block's
+        // next tile is in flight while its threads expand and evaluate the
+        // current one.  The last tile copies rows * Lb rounded up to 16 bytes
+        // (compact allocations are padded, up.h).
+        int tile_bytes = 0;
+        k << "    extern __shared__ __align__(128) unsigned char cdyn[];\n";
         for (size_t c = 0; c < cols.size(); ++c) {
             if (!used[c] || cols[c].Lb == 0) continue;
-            k << "    __shared__ __align__(16) u32 cs" << c << "[" << (256 * R * cols[c].Lb) / 4 + 4 << "];\n";
+            const int words = ((256 * R * cols[c].Lb) / 4 + 4 + 31) / 32 * 32;   // + pad for the expand's look-ahead
+            k << "    u32 *const cs" << c << "_0 = reinterpret_cast<u32 *>(cdyn) + " << tile_bytes / 4
+              << ", *const cs" << c << "_1 = reinterpret_cast<u32 *>(cdyn) + " << tile_bytes / 4 + words << ";\n";
+            tile_bytes += 2 * 4 * words;
         }
+        info.dyn_smem = tile_bytes;
+        k << "    __shared__ __align__(8) u64 cmb[2];\n";
         k << "    constexpr long long TILE = 256 * R;\n";
-        k << "    for (long long t0 = (long long)blockIdx.x * TILE; t0 < n; t0 += (long long)gridDim.x * TILE) {\n";
+        k << "    const long long ntiles = (n + TILE - 1) / TILE;\n";
+        k << "    if (threadIdx.x == 0) { mbar_init(&cmb[0], 1); mbar_init(&cmb[1], 1); mbar_fence_init(); }\n";
+        k << "    __syncthreads();\n";
+        // issue(tile, stage): one thread, all compact columns of the tile
+        k << "    auto issue = [&](long long tile, int st) {\n";
+        k << "        const long long t0 = tile * TILE; const long long rows = n - t0 < TILE ? n - t0 : TILE;\n";
+        k << "        u32 total = 0;\n";
         for (size_t c = 0; c < cols.size(); ++c) {
             if (!used[c] || cols[c].Lb == 0) continue;
-            const int Lb = cols[c].Lb;
-            k << "        { const uint4 *src = reinterpret_cast<const uint4 *>(reinterpret_cast<const unsigned char *>(P.col[" << c
-              << "]) + t0 * " << Lb << ");\n";
-            k << "          const int nv = (int)(((n - t0 < TILE ? n - t0 : TILE) * " << Lb << " + 15) / 16);\n";
-            k << "          for (int i = threadIdx.x; i < nv; i += 256) reinterpret_cast<uint4 *>(cs" << c << ")[i] = __ldcs(src + i); }\n";
+            k << "        const u32 nb" << c << " = (u32)((rows * " << cols[c].Lb << " + 15) / 16 * 16); total += nb" << c << ";\n";
         }
-        k << "        __syncthreads();\n";
-        k << "        const long long base = t0 + (long long)threadIdx.x * R;\n";
+        k << "        mbar_expect_tx(&cmb[st], total);\n";
+        for (size_t c = 0; c < cols.size(); ++c) {
+            if (!used[c] || cols[c].Lb == 0) continue;
+            k << "        bulk_g2s(st ? cs" << c << "_1 : cs" << c << "_0, reinterpret_cast<const unsigned char *>(P.col[" << c << "]) + t0 * "
+              << cols[c].Lb << ", nb" << c << ", &cmb[st]);\n";
+        }
+        k << "    };\n";
+        k << "    if (threadIdx.x == 0 && (long long)blockIdx.x < ntiles) issue(blockIdx.x, 0);\n";
+        k << "    int it = 0;\n";
+        k << "    for (long long tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++it) {\n";
+        k << "        const int st = it & 1;\n";
+        k << "        if (threadIdx.x == 0 && tile + gridDim.x < ntiles) { fence_proxy_async_smem(); issue(tile + gridDim.x, st ^ 1); }\n";
+        k << "        mbar_wait_parity(&cmb[st], (u32)(it >> 1) & 1u);\n";
+        k << "        const long long base = tile * TILE + (long long)threadIdx.x * R;\n";
+        k << "        const bool live = base < n;\n";
     } else {
         k << "    const long long stride = (long long)gridDim.x * blockDim.x * R;\n";
         k << "    for (long long base = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * R; base < n; base += stride) {\n";
+        k << "        const bool live = true;\n";
     }
     for (size_t c = 0; c < cols.size(); ++c) {
         if (!used[c] || cols[c].Lb == 0) continue;
@@ -329,7 +355,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
         const int NW = (R * Lb + 3) / 4 + 1;
         k << "        u32 x" << c << "[R][" << Lc << "];\n";
         k << "        { const int b0 = (int)threadIdx.x * " << R * Lb << ";\n";
-        k << "          const u32 *w = cs" << c << " + (b0 >> 2); const u32 sh0 = (u32)(b0 & 3) * 8u;\n";
+        k << "          const u32 *w = (st ? cs" << c << "_1 : cs" << c << "_0) + (b0 >> 2); const u32 sh0 = (u32)(b0 & 3) * 8u;\n";
         k << "          u32 wv[" << NW + 1 << "];\n";
         k << "#pragma unroll\n          for (int i = 0; i < " << NW + 1 << "; ++i) wv[i] = w[i];\n";
         k << "          u32 al[" << NW << "];   // the thread's bytes, word-aligned\n";
@@ -359,8 +385,8 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     for (size_t c = 0; c < cols.size(); ++c) {
         if (!used[c] || E.lazy[c] || cols[c].Lb > 0) continue;
         const int Lc = cols[c].limbs;
-        k << "        u32 x" << c << "[R][" << Lc << "];\n";
-        k << "        { const u32 *p = P.col[" << c << "] + base; const long long ld = P.ld[" << c << "];\n";
+        k << "        u32 x" << c << "[R][" << Lc << "] = {};\n";
+        k << "        if (live) { const u32 *p = P.col[" << c << "] + base; const long long ld = P.ld[" << c << "];\n";
         if (R == 4) {
             k << "#pragma unroll\n          for (int j = 0; j < " << Lc << "; ++j) { const uint4 v = __ldcs(reinterpret_cast<const uint4 *>(p + j * ld));"
                  " x" << c << "[0][j] = v.x; x" << c << "[1][j] = v.y; x" << c << "[2][j] = v.z; x" << c << "[3][j] = v.w; } }\n";
@@ -370,7 +396,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     }
     const bool store = !opt.sum && !opt.cmp;
     if (store) k << "        u32 res[R][" << LOUT << "];\n";
-    k << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n";
+    k << "#pragma unroll\n        for (int r = 0; r < (live ? R : 0); ++r) {\n";
     k << "            u32 fr = 0; u32 v[" << LOUT << "];\n";
     k << "            eval_row(";
     first = true;
@@ -393,9 +419,9 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     k << "        }\n";
     if (store) {
         if (R == 4)
-            k << "#pragma unroll\n        for (int j = 0; j < " << LOUT << "; ++j) __stcs(reinterpret_cast<uint4 *>(P.out + j * P.ld_out + base), make_uint4(res[0][j], res[1][j], res[2][j], res[3][j]));\n";
+            k << "        if (live)\n#pragma unroll\n        for (int j = 0; j < " << LOUT << "; ++j) __stcs(reinterpret_cast<uint4 *>(P.out + j * P.ld_out + base), make_uint4(res[0][j], res[1][j], res[2][j], res[3][j]));\n";
         else
-            k << "#pragma unroll\n        for (int j = 0; j < " << LOUT << "; ++j) __stcs(P.out + j * P.ld_out + base, res[0][j]);\n";
+            k << "        if (live)\n#pragma unroll\n        for (int j = 0; j < " << LOUT << "; ++j) __stcs(P.out + j * P.ld_out + base, res[0][j]);\n";
     }
     if (any_compact) k << "        __syncthreads();\n";
     k << "    }\n";

@@ -193,6 +193,105 @@ __global__ void __launch_bounds__(256) k_to_compact(const u32 *__restrict__ plan
     }
 }
 
+// Multi-rank combine of grouped aggregates (NEXT-4; aggregate typing
+// P:L1069-1080).  parts: nranks x part_words u32, each rank's output of
+// up_group_aggregate run with AVG replaced by SUM (its partial state); counts:
+// nranks x G row counts.  One thread per (aggregate, group):
+//   SUM  -- exact two's-complement sum over ranks;
+//   MIN / MAX -- signed multi-limb min / max over the ranks whose group is non-empty;
+//   AVG  -- trunc(|SUM| 10^4 / COUNT) sign(SUM) of the combined SUM and COUNT
+//           (reading Q4 truncation; COUNT 0 -> 0).
+struct AggDesc {
+    int kind, Lp, Lr, pad;
+    long long poff, roff;
+};
+__global__ void __launch_bounds__(128) k_group_combine(const u32 *__restrict__ parts, int nranks, long long part_words,
+                                                       const unsigned long long *__restrict__ counts, int G, int n_aggs,
+                                                       const AggDesc *__restrict__ d, u32 *__restrict__ out,
+                                                       unsigned long long *__restrict__ counts_out) {
+    const long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t < G && counts_out) {
+        unsigned long long c = 0;
+        for (int r = 0; r < nranks; ++r) c += counts[(long long)r * G + t];
+        counts_out[t] = c;
+    }
+    if (t >= (long long)G * n_aggs) return;
+    const int a = (int)(t / G), g = (int)(t % G);
+    const AggDesc ad = d[a];
+    u32 *o = out + ad.roff + (long long)g * ad.Lr;
+    unsigned long long cnt = 0;
+    for (int r = 0; r < nranks; ++r) cnt += counts[(long long)r * G + g];
+    if (ad.kind == 1 || ad.kind == 2) {   // MIN / MAX over non-empty ranks
+        int best = -1;
+        for (int r = 0; r < nranks; ++r) {
+            if (counts[(long long)r * G + g] == 0) continue;
+            if (best < 0) { best = r; continue; }
+            const u32 *x = parts + (long long)r * part_words + ad.poff + (long long)g * ad.Lp;
+            const u32 *y = parts + (long long)best * part_words + ad.poff + (long long)g * ad.Lp;
+            int cmp = 0;   // signed compare x vs y
+            if ((int)x[ad.Lp - 1] != (int)y[ad.Lp - 1]) cmp = (int)x[ad.Lp - 1] < (int)y[ad.Lp - 1] ? -1 : 1;
+            for (int j = ad.Lp - 2; j >= 0 && cmp == 0; --j)
+                if (x[j] != y[j]) cmp = x[j] < y[j] ? -1 : 1;
+            if ((ad.kind == 1 && cmp < 0) || (ad.kind == 2 && cmp > 0)) best = r;
+        }
+        for (int j = 0; j < ad.Lr; ++j)
+            o[j] = best < 0 ? 0u : parts[(long long)best * part_words + ad.poff + (long long)g * ad.Lp + (j < ad.Lp ? j : ad.Lp - 1)];
+        return;
+    }
+    // SUM over ranks (Lp limbs, two's complement), kept in up to 80 limbs
+    constexpr int MAXL = 80;
+    u32 acc[MAXL];
+    const int L = ad.Lp < MAXL ? ad.Lp : MAXL;
+    for (int j = 0; j < L; ++j) acc[j] = 0u;
+    for (int r = 0; r < nranks; ++r) {
+        const u32 *x = parts + (long long)r * part_words + ad.poff + (long long)g * ad.Lp;
+        u64 c = 0;
+        for (int j = 0; j < L; ++j) {
+            const u64 v = (u64)acc[j] + x[j] + c;
+            acc[j] = (u32)v;
+            c = v >> 32;
+        }
+    }
+    if (ad.kind == 0) {
+        for (int j = 0; j < ad.Lr; ++j) o[j] = j < L ? acc[j] : ((acc[L - 1] >> 31) ? 0xFFFFFFFFu : 0u);
+        return;
+    }
+    // AVG: |S| 10^4 / COUNT, truncated, with the sign of S
+    const u32 ng = acc[L - 1] >> 31;
+    u32 mag[MAXL + 1];
+    {
+        u64 c = ng;
+        for (int j = 0; j < L; ++j) {
+            const u64 v = (u64)(acc[j] ^ (0u - ng)) + c;
+            mag[j] = (u32)v;
+            c = v >> 32;
+        }
+        u64 m = 0;   // x 10^4
+        for (int j = 0; j < L; ++j) {
+            const u64 v = (u64)mag[j] * 10000u + m;
+            mag[j] = (u32)v;
+            m = v >> 32;
+        }
+        mag[L] = (u32)m;
+    }
+    if (cnt == 0) {
+        for (int j = 0; j < ad.Lr; ++j) o[j] = 0u;
+        return;
+    }
+    unsigned __int128 rem = 0;
+    for (int j = L; j >= 0; --j) {
+        const unsigned __int128 cur = (rem << 32) | mag[j];
+        mag[j] = (u32)(cur / cnt);
+        rem = cur % cnt;
+    }
+    u64 c = ng;
+    for (int j = 0; j < ad.Lr; ++j) {
+        const u64 v = (u64)((j <= L ? mag[j] : 0u) ^ (0u - ng)) + c;
+        o[j] = (u32)v;
+        c = v >> 32;
+    }
+}
+
 int grid_for(long long n, int threads) {
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
@@ -237,6 +336,15 @@ cudaError_t upk_launch_from_compact(const uint8_t *bytes, int Lb, long long n, c
 cudaError_t upk_launch_to_compact(const uint32_t *planes, int L, long long ld, long long n, uint8_t *bytes, int Lb,
                                  cudaStream_t st) {
     k_to_compact<<<grid_for(n, 256), 256, 0, st>>>(planes, L, ld, n, bytes, Lb);
+    return cudaGetLastError();
+}
+
+cudaError_t upk_launch_group_combine(const uint32_t *parts, int nranks, long long part_words,
+                                     const unsigned long long *counts, int G, int n_aggs, const void *d_descs,
+                                     uint32_t *out, unsigned long long *counts_out, cudaStream_t st) {
+    const long long nt = (long long)G * n_aggs > G ? (long long)G * n_aggs : G;
+    k_group_combine<<<(int)((nt + 127) / 128), 128, 0, st>>>(parts, nranks, part_words, counts, G, n_aggs,
+                                                             (const AggDesc *)d_descs, out, counts_out);
     return cudaGetLastError();
 }
 

@@ -370,7 +370,8 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
         kmax += 2;
     }
     int G = G_req;
-    if (G <= 0) G = W <= 64 ? 2 : W <= 160 ? 2 : W <= 700 ? 8 : 32;
+    // lanes per row (measured, profiles/r02_s2-s3): P = 5000 (W = 520) G = 16, P = 20000 G = 32
+    if (G <= 0) G = W <= 160 ? 4 : W <= 700 ? 16 : 32;
     if (G != 1 && G != 2 && G != 4 && G != 8 && G != 16 && G != 32) { err = "band sine: G must divide 32"; return ""; }
     const int R = 32 / G;
     const int KT = kmax + G + 2;

@@ -43,6 +43,9 @@ int upk_contract_tc_slots(int La, int Lb);
 cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, const uint32_t *B, long long ldb, int Lb,
                                    long long n, int sign, unsigned long long *ws, uint32_t *ticket, uint32_t *result,
                                    int LA, int num_sms, cudaStream_t st);
+cudaError_t upk_launch_group_combine(const uint32_t *parts, int nranks, long long part_words,
+                                     const unsigned long long *counts, int G, int n_aggs, const void *d_descs,
+                                     uint32_t *out, unsigned long long *counts_out, cudaStream_t st);
 cudaError_t upk_launch_from_compact(const uint8_t *bytes, int Lb, long long n, const uint32_t *bound, int L,
                                    uint32_t *out, long long ld, uint32_t *flags, cudaStream_t st);
 cudaError_t upk_launch_to_compact(const uint32_t *planes, int L, long long ld, long long n, uint8_t *bytes, int Lb,
@@ -1087,6 +1090,36 @@ up_status up_agg_type(const char *expr, int32_t kind, const up_column *cols, int
     if (p) *p = pp;
     if (s) *s = ss;
     if (limbs) *limbs = limbs_for_precision(pp);
+    return UP_OK;
+}
+
+up_status up_group_combine(up_ctx *c, int32_t n_aggs, const int32_t *kinds, const char *const *exprs,
+                           const up_column *cols, int ncols, int32_t n_groups, int64_t n_global, const uint32_t *d_parts,
+                           int32_t nranks, const uint64_t *d_counts, uint32_t *d_out, uint64_t *d_counts_out,
+                           void *stream) {
+    if (!c || !cols || ncols < 1 || !d_parts || !d_counts || !d_out || nranks < 1)
+        return fail(UP_E_INVAL, "need a ctx, columns, partials, counts and d_out");
+    if (n_aggs < 1 || n_aggs > 32 || !kinds) return fail(UP_E_INVAL, "need 1..32 aggregates");
+    const long long N = n_global > 0 ? n_global : cols[0].n;
+    std::vector<int32_t> pk((size_t)n_aggs);
+    for (int a = 0; a < n_aggs; ++a) pk[(size_t)a] = kinds[a] == AGG_AVG ? AGG_SUM : kinds[a];
+    AggPlan pp, pf;
+    if (up_status s = agg_plan(n_aggs, pk.data(), exprs, cols, ncols, N, n_groups, pp)) return s;
+    if (up_status s = agg_plan(n_aggs, kinds, exprs, cols, ncols, N, n_groups, pf)) return s;
+    struct Desc { int kind, Lp, Lr, pad; long long poff, roff; };
+    std::vector<Desc> d((size_t)n_aggs);
+    for (int a = 0; a < n_aggs; ++a) {
+        d[(size_t)a] = {kinds[a], pp.items[(size_t)a].Lr, pf.items[(size_t)a].Lr, 0, pp.items[(size_t)a].off,
+                        pf.items[(size_t)a].off};
+        if (d[(size_t)a].Lp > 80) return fail(UP_E_UNSUPPORTED, "group_combine: aggregate wider than 80 limbs");
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    std::lock_guard<std::mutex> g(c->mu);
+    if (up_status s = ensure_stage(c, sizeof(Desc) * d.size(), st)) return s;
+    CUDA_TRY(cudaMemcpyAsync(c->d_stage, d.data(), sizeof(Desc) * d.size(), cudaMemcpyHostToDevice, st));
+    CUDA_TRY(upk_launch_group_combine(d_parts, nranks, pp.words, (const unsigned long long *)d_counts, n_groups, n_aggs,
+                                      c->d_stage, d_out, (unsigned long long *)d_counts_out, st));
+    c->launches++;
     return UP_OK;
 }
 

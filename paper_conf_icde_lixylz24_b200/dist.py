@@ -88,3 +88,44 @@ class ShardedSum:
     def result(self) -> str:
         from . import up
         return up.result_to_string(self.result_tensor(), self.S)
+
+
+class ShardedGroupAggregate:
+    """SELECT agg(expr), ... GROUP BY g over a row-sharded table (NEXT-4 across
+    ranks): each rank runs the one-launch grouped aggregation over its rows
+    with AVG computed as SUM (typing with the global row count), one
+    all-gather of the packed partials and one of the group counts, then
+    libup's up_group_combine kernel (exact SUM, MIN / MAX over non-empty
+    ranks, AVG from the combined SUM and COUNT) -- identical on every rank."""
+
+    def __init__(self, ctx, aggs, cols, group, n_groups: int, n_global: int, group_pg=None, stage_host=None):
+        import torch
+        import torch.distributed as dist
+        self.ctx, self.aggs, self.cols, self.group = ctx, list(aggs), list(cols), group
+        self.n_groups, self.n_global, self.pg = n_groups, n_global, group_pg
+        self.world = dist.get_world_size(group_pg) if dist.is_initialized() else 1
+        if stage_host is None:
+            stage_host = dist.is_initialized() and dist.get_backend(group_pg) == "gloo"
+        self.stage_host = stage_host
+
+    def __call__(self):
+        import torch
+        import torch.distributed as dist
+        out, counts, layout = self.ctx.group_aggregate(self.aggs, self.cols, self.group, self.n_groups,
+                                                       self.n_global, partial=self.world > 1)
+        if self.world == 1:
+            return out, counts, layout
+        W = self.world
+        if self.stage_host:
+            ho, hc = out.cpu(), counts.cpu()
+            go = torch.empty(W * ho.numel(), dtype=ho.dtype)
+            gc = torch.empty(W * hc.numel(), dtype=hc.dtype)
+            dist.all_gather_into_tensor(go, ho, group=self.pg)
+            dist.all_gather_into_tensor(gc, hc, group=self.pg)
+            go, gc = go.to(out.device), gc.to(out.device)
+        else:
+            go = torch.empty(W * out.numel(), dtype=out.dtype, device=out.device)
+            gc = torch.empty(W * counts.numel(), dtype=counts.dtype, device=counts.device)
+            dist.all_gather_into_tensor(go, out, group=self.pg)
+            dist.all_gather_into_tensor(gc, counts, group=self.pg)
+        return self.ctx.group_combine(self.aggs, self.cols, go, gc, W, self.n_groups, self.n_global)

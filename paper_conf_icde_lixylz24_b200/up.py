@@ -40,7 +40,7 @@ EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_l
            "up_jit_ms", "up_gen_source", "up_nvrtc_compile", "up_gen_modexp_source", "up_jit_prewarm", "up_gen_sin_source", "up_compact_bytes",
            "up_column_from_host_compact", "up_column_from_device_compact", "up_column_to_host_compact",
            "up_expr_optimized", "up_gen_contract_source", "up_agg_type", "up_group_aggregate",
-           "up_gen_group_agg_source", "up_filter", "up_group_ids"]
+           "up_gen_group_agg_source", "up_filter", "up_group_ids", "up_group_combine"]
 
 AGG = {"SUM": 0, "MIN": 1, "MAX": 2, "AVG": 3}
 
@@ -100,6 +100,8 @@ def lib():
                                           c.c_int64, c.c_char_p, c.c_size_t]
     L.up_filter.argtypes = [P, c.c_char_p, c.c_char_p, c.c_char_p, PC, c.c_int, P, P]
     L.up_group_ids.argtypes = [P, PC, c.c_int, P, c.POINTER(c.c_int64), P, P]
+    L.up_group_combine.argtypes = [P, c.c_int32, PI32, c.POINTER(c.c_char_p), PC, c.c_int, c.c_int32, c.c_int64, P,
+                                   c.c_int32, P, P, P, P]
     L.up_gen_modexp_source.argtypes = [c.c_char_p, c.c_char_p, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
     _lib = L
     return L
@@ -400,13 +402,16 @@ class Context:
         return out
 
     def group_aggregate(self, aggs: Sequence[tuple], cols: Sequence[Column], group=None, n_groups: int = 1,
-                        n_global: int = 0, out=None, counts=None, stream=None):
+                        n_global: int = 0, out=None, counts=None, stream=None, partial: bool = False):
         """SELECT agg(expr), ... GROUP BY group in one launch (include/up.h
         up_group_aggregate).  aggs: [(kind, expr)], kind in AGG's keys.
         Returns (packed int32 device tensor, int64 device counts, layout) where
         layout[a] = (p, s, limbs, offset) and aggregate a of group g occupies
-        out[offset + g*limbs : offset + (g+1)*limbs]."""
+        out[offset + g*limbs : offset + (g+1)*limbs].  partial=True: each AVG
+        is computed as its SUM (the state up_group_combine merges across ranks)."""
         import torch
+        if partial:
+            aggs = [("SUM" if k == "AVG" else k, e) for k, e in aggs]
         layout, off = [], 0
         for kind, expr in aggs:
             p, s, L = agg_type(kind, expr, [(c.p, c.s) for c in cols], n_global or cols[0].n)
@@ -422,6 +427,30 @@ class Context:
                                       group.data_ptr() if group is not None else None, n_groups, n_global,
                                       out.data_ptr(), counts.data_ptr(), _stream_ptr(stream)))
         return out, counts, layout
+
+    def group_combine(self, aggs: Sequence[tuple], cols: Sequence[Column], parts, counts, nranks: int,
+                      n_groups: int = 1, n_global: int = 0, out=None, counts_out=None, stream=None):
+        """Merge nranks gathered group_aggregate(partial=True) outputs (parts:
+        int32 device tensor, rank-major; counts: int64 device tensor nranks x
+        n_groups) into the final aggregates (include/up.h up_group_combine).
+        Returns (packed int32 device tensor, int64 counts, layout) like group_aggregate."""
+        import torch
+        N = n_global or cols[0].n
+        layout, off = [], 0
+        for kind, expr in aggs:
+            p, s, L = agg_type(kind, expr, [(c.p, c.s) for c in cols], N)
+            layout.append((p, s, L, off))
+            off += n_groups * L
+        dev = parts.device
+        if out is None:
+            out = torch.empty(max(off, 1), dtype=torch.int32, device=dev)
+        if counts_out is None:
+            counts_out = torch.empty(n_groups, dtype=torch.int64, device=dev)
+        kinds, exprs = _agg_args(aggs)
+        _chk(lib().up_group_combine(self.h, len(aggs), kinds, exprs, _descs(cols), len(cols), n_groups, N,
+                                    parts.data_ptr(), nranks, counts.data_ptr(), out.data_ptr(), counts_out.data_ptr(),
+                                    _stream_ptr(stream)))
+        return out, counts_out, layout
 
     def filter(self, lhs: str, op: str, rhs: str, cols: Sequence[Column], ids=None, stream=None):
         """WHERE lhs <op> rhs (include/up.h up_filter): rows whose predicate is

@@ -46,6 +46,25 @@ def _worker(rank, world, port, kind, n, q):
         N, _, _ = synth.rsa_modulus(256)
         mag, neg = gdev.uniform_range(synth.SEED, synth.stream_id(4, 0), hi - lo, 0, N - 1, signed=False, row0=lo)
         ss = ShardedSum.modexp(ctx, ctx.column_from_device_bin(len(str(N)), 0, mag, neg), 65537, N, n)
+    elif kind == "group":
+        import numpy as np
+        from paper_conf_icde_lixylz24_b200.dist import ShardedGroupAggregate
+        types = [(12, 2), (12, 2), (3, 2)]
+        cols = [ctx.column_from_host_bin(p, s, *synth.uniform_decimal(hi - lo, p, 8, k + 1, row0=lo))
+                for k, (p, s) in enumerate(types)]
+        gid = torch.as_tensor(_group_ids(n)[lo:hi].copy(), device="cuda")
+        sga = ShardedGroupAggregate(ctx, GROUP_AGGS, cols, gid, 5, n)
+        out, counts, layout = sga()
+        ctx.check()
+        res, cnt = up.group_results(out, counts, layout, 5)
+        allg = [None] * world
+        dist.all_gather_object(allg, (res, cnt))
+        assert all(a == allg[0] for a in allg)
+        if rank == 0:
+            q.put((res, cnt))
+        dist.barrier()
+        dist.destroy_process_group()
+        return
     else:
         mag, neg = synth.normal_decimal(hi - lo, 0.78, 0.01, 8, config=5, column=0, row0=lo)
         ss = ShardedSum.sin(ctx, ctx.column_from_host_bin(9, 8, mag, neg), 300, n)
@@ -62,9 +81,25 @@ def _worker(rank, world, port, kind, n, q):
     dist.destroy_process_group()
 
 
+GROUP_AGGS = [("SUM", "c1"), ("AVG", "c2*(1-c3)"), ("MIN", "c1-c2"), ("MAX", "c2"), ("AVG", "c3")]
+
+
+def _group_ids(n):
+    import numpy as np
+    g = np.random.default_rng(23).integers(0, 5, n).astype(np.int32)
+    g[np.random.default_rng(24).random(n) < 0.1] = -1
+    return g
+
+
 def _oracle_whole(kind, n):
     import oracle
     from gen import synth
+    if kind == "group":
+        types = [(12, 2), (12, 2), (3, 2)]
+        host = [synth.uniform_decimal(n, p, 8, k + 1) for k, (p, s) in enumerate(types)]
+        res, cnt, _ = oracle.group_aggregate(GROUP_AGGS, [oracle.Column(p, s, m, g) for (m, g), (p, s) in zip(host, types)],
+                                             _group_ids(n), 5, n)
+        return (res, cnt)
     if kind == "expr":
         types = [(35, 5), (32, 2)]
         host = [synth.uniform_decimal(n, p, 2, k + 1) for k, (p, s) in enumerate(types)]
@@ -79,7 +114,8 @@ def _oracle_whole(kind, n):
 
 
 @pytest.mark.parametrize("kind,n,world", [("expr", 1, 2), ("expr", 100_003, 2), ("modexp", 3001, 2),
-                                          ("sin", 2049, 2), ("expr", 50_000, 3)])
+                                          ("sin", 2049, 2), ("expr", 50_000, 3), ("group", 30_001, 2),
+                                          ("group", 7, 3)])
 def test_sharded_sum_two_processes_one_gpu(kind, n, world):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")

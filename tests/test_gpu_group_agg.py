@@ -107,3 +107,45 @@ def test_repeat_launches_are_deterministic():
     a = _check(Q1_AGGS + [("MIN", "c2*(1-c3)"), ("MAX", "c1")], host, types, gid, 4)
     b = _check(Q1_AGGS + [("MIN", "c2*(1-c3)"), ("MAX", "c1")], host, types, gid, 4)
     assert bool((a == b).all())
+
+
+@pytest.mark.parametrize("nranks", [2, 3, 5])
+@pytest.mark.parametrize("case", ["q1", "wide"])
+def test_multi_rank_group_combine(nranks, case):
+    """Row shards' group_aggregate(partial=True) (AVG as SUM, global-N typing),
+    concatenated rank-major as an all-gather would, merged by up_group_combine
+    == the oracle's whole-table aggregates (includes groups empty on some
+    ranks: with 7 groups and 200 rows over 5 shards)."""
+    import torch
+    from paper_conf_icde_lixylz24_b200 import up
+    if case == "q1":
+        types, aggs, n, ng = [(12, 2), (12, 2), (3, 2), (3, 2)], Q1_AGGS + [("MIN", "c1"), ("MAX", "c2*(1-c3)")], 6007, 4
+        host = G.gen_cols(n, types, config=8)
+    else:
+        types, n, ng = [(60, 10), (45, 5)], 200, 7
+        aggs = [(k, e) for e in ("c1*c2", "c1/c2") for k in ("SUM", "MIN", "MAX", "AVG")]
+        host = G.gen_cols(n, types, config=8, nonzero_lead_cols=(1,), seed=11)
+    gid = _gid(n, ng, 17)
+    c = G.ctx()
+    parts, cnts = [], []
+    for r in range(nranks):
+        lo, hi = n * r // nranks, n * (r + 1) // nranks
+        sh = [(m[lo:hi], g[lo:hi]) for m, g in host]
+        gcols = G.to_gpu(sh, types) if hi > lo else [c.column_from_host_bin(p, s, np.zeros((0, 1), np.uint32))
+                                                      for p, s in types]
+        dg = torch.as_tensor(np.ascontiguousarray(gid[lo:hi]), device="cuda")
+        o, k, _ = c.group_aggregate(aggs, gcols, dg if hi > lo else None, ng, n, partial=True) if hi > lo else \
+            (None, None, None)
+        if o is None:
+            continue
+        parts.append(o)
+        cnts.append(k)
+    out, counts, layout = c.group_combine(aggs, G.to_gpu(host, types), torch.cat(parts), torch.cat(cnts), len(parts),
+                                          ng, n)
+    c.check()
+    got, got_counts = up.group_results(out, counts, layout, ng)
+    want, want_counts, want_types = oracle.group_aggregate(aggs, G.to_oracle(host, types), gid, ng, n)
+    assert [(p, s) for p, s, _, _ in layout] == want_types
+    assert got_counts == want_counts
+    for a, (g_a, w_a) in enumerate(zip(got, want)):
+        assert g_a == w_a, f"aggregate {a} {aggs[a]}"

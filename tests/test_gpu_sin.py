@@ -135,3 +135,28 @@ def test_sin_v2_kernels_still_exact(P, monkeypatch):
     out = c.sin_taylor(x, P)
     c.check()
     assert c.column_to_strings(out) == oracle.sin_rows(oracle.Column(9, 8, mag, neg), P)
+
+
+@pytest.mark.parametrize("lanes", [1, 2, 8, 32])
+@pytest.mark.parametrize("P,n", [(8, 100), (60, 300), (300, 70), (1000, 40)])
+@pytest.mark.parametrize("pst", [(9, 8), (8, 7), (3, 2), (1, 0), (9, 9)])
+def test_sin_band_kernel_every_shape(lanes, P, n, pst, monkeypatch):
+    """The skewed-band kernel (sin_band.cpp; default for W > 200 limbs) forced
+    at every P and scale shape: 2s = 16 (the complement trick for negative
+    terms), 2s = 14 / 4 / 0 / 18 (general scaled adds, digit drops at
+    different term parities, whole-digit normalisation shifts sd = 1 for
+    s <= 6), G lanes per row from 1 to 32, rows spanning several warps."""
+    monkeypatch.setenv("UP_SIN_BAND_G", str(lanes))
+    p, s = pst
+    if s > P:
+        pytest.skip("s > P is outside sin_taylor's domain (reading Q20)")
+    mag, neg = synth.uniform_decimal(n, p, 5, 6)
+    c = G.ctx()
+    x = c.column_from_host_bin(p, s, mag, neg)
+    out = c.sin_taylor(x, P)
+    c.check()
+    assert c.column_to_strings(out) == oracle.sin_rows(oracle.Column(p, s, mag, neg), P)
+    from paper_conf_icde_lixylz24_b200 import up
+    res = c.sin_taylor_sum(x, P)
+    c.check()
+    assert up.result_to_string(res, P) == oracle.sin_sum(oracle.Column(p, s, mag, neg), P, threads=8)
