@@ -15,15 +15,10 @@
 
 namespace uph {
 
-// experiment knob: UP_MUL28=1 switches expression multiplies to radix-2^28
-// product scanning (up_dev.cuh mul_mag28).  Measured on B200: cfg3 p = 200
-// 4.41e9 vs 4.66e9 rows/s for the 32-bit operand scanning (kept default),
-// p = 500 +2%.  modexp uses radix 2^28 unconditionally (special.cpp).
-std::string mul_variant_define() { return getenv("UP_MUL28") ? "#define UP_MUL28 1\n" : ""; }
+std::string mul_variant_define() { return ""; }
 
 std::string launch_bounds(int threads, int min_blocks) {
     std::string s = "__launch_bounds__(" + std::to_string(threads);
-    if (const char *m = getenv("UP_MINBLOCKS")) min_blocks = atoi(m);
     if (min_blocks > 0) s += ", " + std::to_string(min_blocks);
     return s + ")";
 }
@@ -50,10 +45,10 @@ int mag_limbs_of_pow10(int k) {   // limbs of the magnitude 10^k - 1 (at least 1
 // so the window only trades speed.  Used when the divisor is wider than the
 // window and the dividend reaches into it.  Returns T, or 0.
 int div_top_window(const Node *n) {
-    if (n->op != Op::Div || getenv("UP_NO_DIVTOP")) return 0;
+    if (n->op != Op::Div) return 0;
     const int La = n->l->L, Lb = n->r->L;
     const int NC = (int)HBig::pow10(n->r->s + 4).w.size();
-    const int T = std::max(NC, n->L) + (getenv("UP_DIVTOP_T2") ? 2 : 1);
+    const int T = std::max(NC, n->L) + 1;
     const int E = Lb - T;
     return (E > 0 && La > E) ? T : 0;
 }
@@ -514,11 +509,6 @@ std::string gen_group_agg_kernel(const std::vector<AggItem> &aggs, const std::ve
         const int nb = std::min<int>({32, 2048 / t, (int)((228u * 1024u) / blk)});
         if (nb >= 1 && per_thread * (size_t)t <= 220 * 1024 && nb * t >= best_threads) { best_threads = nb * t; T = t; }
     }
-    if (const char *e = getenv("UP_GAGG_T")) {   // experiment: force T private records (<= 220 KB)
-        const int t = atoi(e);
-        T = (t == 32 || t == 64 || t == 128 || t == 256) && per_thread * (size_t)t <= 220 * 1024 ? t : 0;
-    }
-    if (getenv("UP_GAGG_WARP")) T = 0;
     const bool priv = T > 0;
     const int R = priv && maxL <= 8 && !divmod ? 4 : 1;
     if (!priv) T = 256;
@@ -1075,157 +1065,6 @@ std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int
     return k.str();
 }
 
-// Row contraction SUM_rows(c_a * c_b) in radix 2^28 (same contract as
-// gen_contract_kernel): the operands' 32-bit limb planes are read as 28-bit
-// digits (two loads + a funnel shift per digit), so every digit product is
-// < 2^56 and the products of one row's column sum in a 64-bit register with
-// one IMAD.WIDE.U32 accumulate each (the 32-bit version needs the product plus
-// two 64-bit adds).  Before each row the column registers are renormalised
-// (lo < 2^62, the overflow counted in hi, units 2^62), so a row's <= 255
-// products (< 2^63.9 in total) never overflow.  Warp w owns digit columns
-// [wK, wK + K) (circular operand window as in gen_contract_kernel); the
-// two's-complement sign corrections stay on 32-bit word positions.
-std::string gen_contract_kernel28(int La, int Lb, int LA, int sign, int col_a, int col_b, GenInfo &info) {
-    const int DA = (32 * La + 27) / 28, DB = (32 * Lb + 27) / 28;
-    const int NK = DA + DB - 1;                   // digit columns of the product
-    const int K = (NK + 7) / 8 <= 16 ? 8 : 16;
-    const int CR = (NK + K - 1) / K;
-    const int NSL = La + Lb + 6;                  // 32-bit slots (a column's 128-bit sum spills into 5 words)
-    if (CR > 16 || DA > 255 || DB > 255 || CR * K < La + Lb + 1) return "";
-    info.threads = CR * 32;
-    info.rows_per_block = 32;
-    info.ws_slots = 2 * NSL;
-    info.dyn_smem = 0;
-    std::ostringstream k;
-    k << "// generated by libup: row contraction (radix 2^28) SUM(c" << col_a + 1 << "*c" << col_b + 1 << ") La=" << La
-      << " Lb=" << Lb << " K=" << K << " ranges=" << CR << "\n";
-    k << mul_variant_define() << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
-    k << "__device__ __forceinline__ u32 dig28(const u32 *X, long long ld, int L, int d, long long row) {\n";
-    k << "    const int b = 28 * d, w = b >> 5, o = b & 31;\n";
-    k << "    const u32 lo = (d >= 0 && w < L) ? __ldg(X + (long long)w * ld + row) : 0u;\n";
-    k << "    const u32 hi = (d >= 0 && w + 1 < L) ? __ldg(X + (long long)(w + 1) * ld + row) : 0u;\n";
-    k << "    return __funnelshift_r(lo, hi, (u32)o) & M28;\n}\n";
-    // branch-free guarded load: always load (from the row's own first word when
-    // out of range, a valid address), then select
-    k << "__device__ __forceinline__ u32 ldsel(bool ok, const u32 *p, const u32 *safe) {\n";
-    k << "    const u32 v = __ldg(ok ? p : safe); return ok ? v : 0u;\n}\n\n";
-    k << "extern \"C\" __global__ void __launch_bounds__(" << CR * 32 << ") upk(const up_kparams P) {\n";
-    k << "    constexpr int LA_ = " << La << ", LB_ = " << Lb << ", DA = " << DA << ", DB = " << DB << ", K = " << K
-      << ", NSL = " << NSL << ";\n";
-    k << "    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n";
-    k << "    const int k0 = warp * K;   // digit columns [k0, k0+K); 32-bit correction words [k0, k0+K)\n";
-    k << "    const u32 *A = P.col[" << col_a << "], *B = P.col[" << col_b << "];\n";
-    k << "    const long long lda = P.ld[" << col_a << "], ldb = P.ld[" << col_b << "];\n";
-    k << "    u64 lo[K], cor[K]; u32 hi[K]; u64 ss = 0;\n";
-    k << "#pragma unroll\n    for (int m = 0; m < K; ++m) { lo[m] = 0ull; hi[m] = 0u; cor[m] = 0ull; }\n";
-    k << "    const int ilo = k0 - (DB - 1) > 0 ? k0 - (DB - 1) : 0;\n";
-    k << "    const int ihi = k0 + K - 1 < DA - 1 ? k0 + K - 1 : DA - 1;\n";
-    k << "    const int ib0 = ilo - ilo % K;\n";
-    k << "    const long long n = P.n;\n";
-    k << "    for (long long r0 = (long long)blockIdx.x * 32; r0 < n; r0 += (long long)gridDim.x * 32) {\n";
-    k << "        const long long row = r0 + lane;\n";
-    k << "        if (row < n) {\n";
-    k << "#pragma unroll\n            for (int m = 0; m < K; ++m) { hi[m] += (u32)(lo[m] >> 62); lo[m] &= 0x3FFFFFFFFFFFFFFFull; }\n";
-    // digit d starts at bit 28 d; for d = 8t + u the word is 7t + (28u >> 5) and
-    // the shift (28u & 31): K-blocks start at multiples of 8 (k0, ib0 are), so
-    // every offset and shift below is static and only 7t moves per block
-    k << "            if (ilo <= ihi) {\n";
-    k << "            const u32 *Ar = A + row, *Br = B + row;\n";
-    k << "            u32 c[K];\n";
-    k << "            { const int jb = k0 - ib0;   // window digits jb + m, jb a multiple of 8\n";
-    k << "              const u32 *pb = Br + (long long)((jb >> 3) * 7) * ldb;\n";
-    k << "#pragma unroll\n              for (int m = 0; m < K; ++m) {\n";
-    k << "                const int j = jb + m, w = (jb >> 3) * 7 + ((28 * m) >> 5);\n";
-    k << "                const u32 lo = ldsel(j >= 0 && j < DB && w >= 0 && w < LB_, pb + (long long)((28 * m) >> 5) * ldb, Br);\n";
-    k << "                const u32 hi = ldsel(j >= 0 && j < DB && w + 1 >= 0 && w + 1 < LB_, pb + (long long)(((28 * m) >> 5) + 1) * ldb, Br);\n";
-    k << "                c[m] = __funnelshift_r(lo, hi, (u32)((28 * m) & 31)) & M28; } }\n";
-    k << "            for (int ib = ib0; ib <= ihi; ib += K) {\n";
-    k << "              const u32 *pa = Ar + (long long)((ib >> 3) * 7) * lda;\n";
-    k << "              const int jb = k0 - ib - 8;   // B digits jb + 7 - u (u = 0..K-1) refill the window\n";
-    k << "              const u32 *pb = Br + (long long)((jb >> 3) * 7) * ldb;\n";
-    k << "#pragma unroll\n              for (int u = 0; u < K; ++u) {\n";
-    k << "                const int i = ib + u, wa = (ib >> 3) * 7 + ((28 * u) >> 5);\n";
-    k << "                const bool ia = i >= ilo && i <= ihi;\n";
-    k << "                const u32 alo = ldsel(ia && wa < LA_, pa + (long long)((28 * u) >> 5) * lda, Ar);\n";
-    k << "                const u32 ahi = ldsel(ia && wa + 1 < LA_, pa + (long long)(((28 * u) >> 5) + 1) * lda, Ar);\n";
-    k << "                const u32 ai = __funnelshift_r(alo, ahi, (u32)((28 * u) & 31)) & M28;\n";
-    k << "#pragma unroll\n                for (int m = 0; m < K; ++m) lo[m] += mulw(ai, c[(m - u + K) % K]);\n";
-    // B digit j = k0 - i - 1 = jb + 7 - u: bits 28 (7 - u) above digit jb's word base
-    k << "                { const int j = jb + 7 - u;\n";
-    k << "                  constexpr int dummy = 0; (void)dummy;\n";
-    k << "                  const int rb = 28 * (7 - u), ow = rb >= 0 ? (rb >> 5) : -((-rb + 31) >> 5), sh = rb - 32 * ow;\n";
-    k << "                  const int w = (jb >> 3) * 7 + ow;\n";
-    k << "                  const bool jv = j >= 0 && j < DB;\n";
-    k << "                  const u32 blo = ldsel(jv && w >= 0 && w < LB_, pb + (long long)ow * ldb, Br);\n";
-    k << "                  const u32 bhi = ldsel(jv && w + 1 >= 0 && w + 1 < LB_, pb + (long long)(ow + 1) * ldb, Br);\n";
-    k << "                  c[K - 1 - u] = __funnelshift_r(blo, bhi, (u32)sh) & M28; }\n";
-    k << "              }\n";
-    k << "            }\n";
-    k << "            }\n";
-    // sign corrections on 32-bit word positions (as gen_contract_kernel)
-    k << "            const u32 sa = __ldg(A + (long long)(LA_ - 1) * lda + row) >> 31;\n";
-    k << "            const u32 sb = __ldg(B + (long long)(LB_ - 1) * ldb + row) >> 31;\n";
-    k << "            if (sa) {\n#pragma unroll\n              for (int m = 0; m < K; ++m) { const int j = k0 + m - LA_; if (j >= 0 && j < LB_) cor[m] += __ldg(B + (long long)j * ldb + row); } }\n";
-    k << "            if (sb) {\n#pragma unroll\n              for (int m = 0; m < K; ++m) { const int j = k0 + m - LB_; if (j >= 0 && j < LA_) cor[m] += __ldg(A + (long long)j * lda + row); } }\n";
-    k << "            ss += sa & sb;\n";
-    k << "        }\n";
-    k << "    }\n";
-    // column value lo + hi 2^62 as a 128-bit (vl, vh), then the warp reduction
-    k << "    u64 vl[K], vh[K];\n";
-    k << "#pragma unroll\n    for (int m = 0; m < K; ++m) { const u64 t = lo[m] + ((u64)hi[m] << 62); vh[m] = (u64)(hi[m] >> 2) + (t < lo[m] ? 1ull : 0ull); vl[m] = t; }\n";
-    k << "#pragma unroll\n    for (int m = 0; m < K; ++m) {\n";
-    k << "#pragma unroll\n        for (int o = 16; o > 0; o >>= 1) {\n";
-    k << "            const u64 l2 = __shfl_down_sync(0xFFFFFFFFu, vl[m], o); const u64 h2 = __shfl_down_sync(0xFFFFFFFFu, vh[m], o);\n";
-    k << "            const u64 s = vl[m] + l2; vh[m] += h2 + (s < l2 ? 1ull : 0ull); vl[m] = s;\n";
-    k << "            cor[m] += __shfl_down_sync(0xFFFFFFFFu, cor[m], o);\n";
-    k << "        }\n    }\n";
-    k << "#pragma unroll\n    for (int o = 16; o > 0; o >>= 1) ss += __shfl_down_sync(0xFFFFFFFFu, ss, o);\n";
-    k << "    u64 *pos = P.ws, *neg = P.ws + NSL;\n";
-    k << "    if (lane == 0) {\n";
-    k << "#pragma unroll\n        for (int m = 0; m < K; ++m) {\n";
-    k << "            const int col = k0 + m;\n";
-    k << "            if (col < DA + DB - 1) {\n";
-    k << "                const int bp = 28 * col, w = bp >> 5; const u32 o = (u32)(bp & 31);\n";
-    k << "                const u32 v[4] = {(u32)vl[m], (u32)(vl[m] >> 32), (u32)vh[m], (u32)(vh[m] >> 32)};\n";
-    k << "#pragma unroll\n                for (int q = 0; q < 5; ++q) {\n";
-    k << "                    const u32 x = __funnelshift_l(q > 0 ? v[q > 0 ? q - 1 : 0] : 0u, q < 4 ? v[q < 4 ? q : 0] : 0u, o);\n";
-    k << "                    if (x && w + q < NSL) atomicAdd(&pos[w + q], (u64)x);\n";
-    k << "                }\n";
-    k << "            }\n";
-    k << "            if (k0 + m + 1 < NSL) {\n";
-    k << "                if ((u32)cor[m]) atomicAdd(&neg[k0 + m], (u64)(u32)cor[m]);\n";
-    k << "                if (cor[m] >> 32) atomicAdd(&neg[k0 + m + 1], cor[m] >> 32);\n";
-    k << "            }\n        }\n";
-    k << "        if (warp == 0 && ss) atomicAdd(&pos[LA_ + LB_], ss);\n";
-    k << "    }\n";
-    // last block: normalise pos - neg into LA limbs (as gen_contract_kernel)
-    k << "    __threadfence();\n    __syncthreads();\n";
-    k << "    __shared__ u32 s_last;\n";
-    k << "    if (threadIdx.x == 0) s_last = (atomicAdd(P.ticket, 1u) == gridDim.x - 1) ? 1u : 0u;\n";
-    k << "    __syncthreads();\n    if (!s_last) return;\n    __threadfence();\n";
-    k << "    __shared__ u64 sp[NSL], sn[NSL];\n";
-    k << "    for (int i = threadIdx.x; i < NSL; i += blockDim.x) { sp[i] = atomicExch(&pos[i], 0ull); sn[i] = atomicExch(&neg[i], 0ull); }\n";
-    k << "    __syncthreads();\n";
-    k << "    if (threadIdx.x == 0) {\n";
-    k << "        *P.ticket = 0u;\n";
-    k << "        u64 cp = 0, cn = 0; u32 borrow = 0, cneg = " << (sign < 0 ? 1 : 0) << "u;\n";
-    k << "        for (int j = 0; j < " << LA << "; ++j) {\n";
-    k << "            u64 tp = cp, tn = cn;\n";
-    k << "            if (j < NSL) { tp += (u32)sp[j]; tn += (u32)sn[j]; }\n";
-    k << "            if (j >= 1 && j - 1 < NSL) { tp += sp[j - 1] >> 32; tn += sn[j - 1] >> 32; }\n";
-    k << "            cp = tp >> 32; cn = tn >> 32;\n";
-    k << "            const u64 d = (u64)(u32)tp - (u32)tn - borrow;\n";
-    k << "            borrow = (u32)(d >> 63);\n";
-    if (sign < 0) {
-        k << "            const u64 ng = (u64)(~(u32)d) + cneg; cneg = (u32)(ng >> 32);\n";
-        k << "            P.result[j] = (u32)ng;\n";
-    } else {
-        k << "            P.result[j] = (u32)d;\n";
-    }
-    k << "        }\n    }\n";
-    k << "}\n";
-    return k.str();
-}
 
 namespace {
 void flatten_any(const Node *n, int sign, std::vector<std::pair<int, const Node *>> &out) {

@@ -34,7 +34,6 @@ struct SplitTerm {
     int sign, col_a, col_b;
 };
 std::string gen_contract_kernel(int La, int Lb, int LA, int sign, int col_a, int col_b, GenInfo &info);
-std::string gen_contract_kernel28(int La, int Lb, int LA, int sign, int col_a, int col_b, GenInfo &info);
 bool split_sum_terms(const Node *root, const std::vector<ColType> &cols, int min_products,
                      std::vector<SplitTerm> &prods, std::unique_ptr<Node> &rest, int &rest_scale);
 // wide SUM regime (warp per row); "" if the expression does not fit it

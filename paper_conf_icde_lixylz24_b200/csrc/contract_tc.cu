@@ -11,11 +11,13 @@
 // P:L576-607 with the row sum of P:L1069-1080 moved inside it, which SUM's
 // linearity allows).  D is one integer GEMM (M = digits of c_a, N = digits
 // of c_b, K = rows) issued as tcgen05.mma kind::i8 with the accumulator in
-// TMEM.  The limb planes are not K-major byte matrices, so the CTA's threads
-// load 16-row x 1-limb pieces (4 x LDG.128), transpose bytes with PRMT and
-// write the canonical no-swizzle K-major core-matrix layout into shared
-// memory (two stages); one thread issues the MMAs and commits them to an
-// mbarrier.  Every <= 32768 rows (255^2 * 32768 < 2^31) the accumulator is
+// TMEM.  A control warp's lane 0 brings each stage's limb-plane boxes (c_a's
+// limbs of the M tile, c_b's of the N group, KC rows) into shared memory with
+// 2-D TMA copies completing on mbarriers; 16 transform warps rewrite them in
+// the canonical MN-major no-swizzle core-matrix layout -- a WORD transpose:
+// the 16 digit bytes of one row in a 16-digit chunk are the little-endian
+// words of 4 consecutive limbs -- and the control lane issues the MMAs and
+// commits them to an mbarrier.  Every <= 32768 rows (255^2 * 32768 < 2^31) the accumulator is
 // drained: each thread reads its TMEM lane (one digit x) and adds D[x][y]
 // into per-CTA anti-diagonal sums (u64, shared memory).  At the end the
 // CTAs add their sums into 32-bit-aligned u64 slots (positive and negative
@@ -473,10 +475,6 @@ cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, con
     const size_t need256 = (size_t)2 * nraw * 256 * 4 + 2 * (size_t)(128 + W) * 256;
     const size_t need128 = (size_t)3 * nraw * 128 * 4 + 2 * (size_t)(128 + W) * 128;   // >= 3 raw stages at 128 rows
     const int max_tasks = (8 + W / 16) * 128;             // transform tasks per 128-row stage (<= 512 x MAXT)
-    if (const char *kc = getenv("UP_TC_KC")) {              // experiments: force the stage depth
-        if (atoi(kc) == 256) return launch_kc<256>(P, W, nraw, num_sms, st);
-        if (atoi(kc) == 64) return launch_kc<64>(P, W, nraw, num_sms, st);
-    }
     if (need256 + 16 * 1024 <= 220 * 1024 && max_tasks * 2 <= 512 * 16) return launch_kc<256>(P, W, nraw, num_sms, st);
     if (need128 + 16 * 1024 <= 220 * 1024 && max_tasks <= 5120) return launch_kc<128>(P, W, nraw, num_sms, st);
     return launch_kc<64>(P, W, nraw, num_sms, st);

@@ -163,12 +163,6 @@ struct up_ctx {
     std::unordered_map<std::string, std::unique_ptr<JitKernel>> by_src;
     std::unordered_map<std::string, JitKernel *> by_key;
     std::unordered_map<std::string, SplitPlan> plans;   // split SUM plans (up_sum_expr)
-    // side stream of a split SUM: the (ALU-bound) rest kernel overlaps the
-    // (HBM-bound) tensor-core contraction; it has its own SUM workspace
-    cudaStream_t side = nullptr;
-    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
-    unsigned long long *d_ws2 = nullptr;
-    uint32_t *d_ticket2 = nullptr;
     uint64_t launches = 0;
     double jit_ms = 0.0;
     std::mutex mu;
@@ -360,8 +354,6 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     if (getenv("UP_NO_OPT")) k += "|noopt";
     if (getenv("UP_NO_WIDE")) k += "|nowide";
     if (getenv("UP_SPLIT")) k += "|split";
-    if (getenv("UP_MUL28")) k += "|mul28";
-    if (const char *m = getenv("UP_MINBLOCKS")) k += std::string("|mb") + m;
     return k;
 }
 
@@ -506,11 +498,6 @@ up_status up_ctx_destroy(up_ctx *c) {
     if (c->d_stage) cudaFree(c->d_stage);
     if (c->d_scratch) cudaFree(c->d_scratch);
     if (c->d_parts) cudaFree(c->d_parts);
-    if (c->d_ws2) cudaFree(c->d_ws2);
-    if (c->d_ticket2) cudaFree(c->d_ticket2);
-    if (c->side) cudaStreamDestroy(c->side);
-    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
-    if (c->ev_join) cudaEventDestroy(c->ev_join);
     delete c;
     return UP_OK;
 }
@@ -802,16 +789,12 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     const long long N = n_global > 0 ? n_global : cols[0].n;
     if (N < cols[0].n) return fail(UP_E_INVAL, "n_global < local rows");
     // Split SUM: top-level column products -> row-contraction kernels, the
-    // rest -> the fused per-thread kernel, then an exact combine (SUM is linear).
-    // opt-in (UP_SPLIT=1): measured slower than the fused per-thread kernel at
-    // p = 200 (7.5 vs 2.9 ms) and only 1.2x faster at p = 1000 in round 1
-    // row-contraction split: forced by UP_SPLIT, automatic when a top-level
-    // column product is at least kSplitAutoProducts limb products (measured on
-    // B200: cfg3 p = 1000 (104 x 104 limbs) 5.9e7 -> 7.2e7 rows/s; p = 500
-    // (52 x 52) and p = 200 stay faster fused), off with UP_NO_SPLIT
-    // With the tensor-core contraction (contract_tc.cu, default; UP_NO_TC for
-    // the CUDA-core one) every top-level column product of >= kContractMinProducts
-    // limb products is split off.
+    // rest -> the fused per-thread kernel, then an exact combine (SUM is
+    // linear).  With the tensor-core contraction (contract_tc.cu, default)
+    // every top-level column product of >= kContractMinProducts limb products
+    // is split off (cfg3 p = 200: 4.4e9 -> 1.1e10 rows/s); the CUDA-core
+    // contraction (UP_NO_TC, and beyond 2^31 rows per call) only from
+    // kSplitAutoProducts.  Test switches: UP_SPLIT forces, UP_NO_SPLIT disables.
     // (TMA row coordinates are 32-bit signed: more rows per call take the CUDA-core contraction)
     const bool use_tc = getenv("UP_NO_TC") == nullptr && cols[0].n < (1ll << 31);
     bool try_split = getenv("UP_SPLIT") != nullptr;
@@ -827,9 +810,7 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     if (try_split && !getenv("UP_NO_SPLIT")) {
         // the split plan (terms, kernels) is cached per (expression, column types, N, knobs):
         // typing, optimising and splitting cost host time on every call otherwise
-        const bool r28 = getenv("UP_CONTRACT28") != nullptr;
-        std::string pkey = key_of("splitplan", expr, cols, ncols, 0) + "|" + std::to_string(N) + (use_tc ? "|tc" : "") +
-                           (r28 ? "|r28" : "");
+        std::string pkey = key_of("splitplan", expr, cols, ncols, 0) + "|" + std::to_string(N) + (use_tc ? "|tc" : "");
         auto pit = c->plans.find(pkey);
         if (pit == c->plans.end()) {
             SplitPlan pl;
@@ -848,13 +829,8 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
                     if (!(use_tc && upk_contract_tc_slots(La, Lb) <= kWsSlots)) {
                         std::string key = "contract|" + std::to_string(La) + "|" + std::to_string(Lb) + "|" + std::to_string(LAs) +
                                           "|" + std::to_string(st.sign) + "|" + std::to_string(st.col_a) + "|" + std::to_string(st.col_b);
-                        // radix-2^28 contraction: opt-in (measured: equal at p = 1000, slower at p = 500)
-                        if (r28) key += "|r28";
                         if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
-                                std::string src;
-                                if (r28) src = gen_contract_kernel28(La, Lb, LAs, st.sign, st.col_a, st.col_b, info);
-                                if (src.empty()) { info = GenInfo(); src = gen_contract_kernel(La, Lb, LAs, st.sign, st.col_a, st.col_b, info); }
-                                return src; }, &kc))
+                                return gen_contract_kernel(La, Lb, LAs, st.sign, st.col_a, st.col_b, info); }, &kc))
                             return s;
                     }
                     pl.cc_kernels.push_back(kc);   // nullptr: tensor-core contraction
@@ -889,15 +865,6 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             P.ticket = c->d_ticket;
             P.flags = c->d_flags;
             int ti = 0;
-            // the rest kernel runs on the side stream, concurrently with the contractions
-            // opt-in (UP_OVERLAP=1): measured slower on B200 (cfg3 p=200 1.42 -> 2.09 ms): one rest
-            // block per SM beside the contraction's CTA is slower than the two kernels back to back
-            const bool overlap = pl.rest_kernel && !pl.prods.empty() && getenv("UP_OVERLAP");
-            if (overlap && c->side) {
-                // fork before the contractions are enqueued: the side stream waits only for earlier work
-                CUDA_TRY(cudaEventRecord(c->ev_fork, (cudaStream_t)stream));
-                CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_fork, 0));
-            }
             for (size_t q = 0; q < pl.prods.size(); ++q) {
                 const SplitTerm &st = pl.prods[q];
                 const up_column &ca = cols[st.col_a], &cb = cols[st.col_b];
@@ -911,36 +878,10 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
                 P.result = c->d_parts + (size_t)ti++ * LAs;
                 if (up_status s = launch(c, pl.cc_kernels[q], P, P.n, (cudaStream_t)stream)) return s;
             }
-            if (overlap) {
-                if (!c->side) {
-                    CUDA_TRY(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
-                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
-                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
-                    CUDA_TRY(cudaMalloc(&c->d_ws2, sizeof(unsigned long long) * kWsSlots));
-                    CUDA_TRY(cudaMemset(c->d_ws2, 0, sizeof(unsigned long long) * kWsSlots));
-                    CUDA_TRY(cudaMalloc(&c->d_ticket2, 64));
-                    CUDA_TRY(cudaMemset(c->d_ticket2, 0, 64));
-                    CUDA_TRY(cudaDeviceSynchronize());
-                    CUDA_TRY(cudaEventRecord(c->ev_fork, (cudaStream_t)stream));   // first use: after the contractions
-                    CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_fork, 0));
-                }
-                up_kparams R = P;
-                R.ws = c->d_ws2;
-                R.ticket = c->d_ticket2;
-                R.result = c->d_parts + (size_t)pl.prods.size() * LAs;
-                // one block per SM: it shares each SM with the contraction's CTA (launched first)
-                const int bps = pl.rest_kernel->blocks_per_sm;
-                pl.rest_kernel->blocks_per_sm = 1;
-                const up_status ls = launch(c, pl.rest_kernel, R, R.n, c->side);
-                pl.rest_kernel->blocks_per_sm = bps;
-                if (ls) return ls;
-                CUDA_TRY(cudaEventRecord(c->ev_join, c->side));
-            }
-            if (pl.rest_kernel && !overlap) {
+            if (pl.rest_kernel) {
                 P.result = c->d_parts + (size_t)ti++ * LAs;
                 if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream)) return s;
             }
-            if (overlap) CUDA_TRY(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_join, 0));
             if (pl.rest_kernel && pl.rest_scale > 0) {
                 const uint32_t *d_sc = nullptr;
                 if (up_status s = pow10_device(c, pl.rest_scale, &d_sc)) return s;
@@ -1052,8 +993,6 @@ up_status agg_plan(int32_t n_aggs, const int32_t *kinds, const char *const *expr
     pl.key = "gagg|" + std::to_string(G) + "|" + std::to_string(N);
     for (int i = 0; i < ncols; ++i) pl.key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
     if (getenv("UP_NO_OPT")) pl.key += "|noopt";
-    if (getenv("UP_GAGG_WARP")) pl.key += "|warp";
-    if (const char *e = getenv("UP_GAGG_T")) pl.key += std::string("|T") + e;
     for (int a = 0; a < n_aggs; ++a) {
         Typed &t = pl.typed[(size_t)a];
         if (up_status st = type_expr(exprs[a], cols, ncols, t)) return st;
@@ -1245,8 +1184,7 @@ up_status up_expr_optimized(const char *expr, const up_column *cols, int ncols, 
 // generated row-contraction source (diagnostics / prewarm)
 up_status up_gen_contract_source(int32_t La, int32_t Lb, int32_t LA, int sign, char *buf, size_t len) {
     GenInfo info;
-    std::string src = getenv("UP_CONTRACT28") ? gen_contract_kernel28(La, Lb, LA, sign, 0, 1, info) : "";
-    if (src.empty()) { info = GenInfo(); src = gen_contract_kernel(La, Lb, LA, sign, 0, 1, info); }
+    const std::string src = gen_contract_kernel(La, Lb, LA, sign, 0, 1, info);
     if (src.empty()) return fail(UP_E_UNSUPPORTED, "no contraction kernel");
     if (src.size() + 1 > len) return fail(UP_E_NOMEM, "buffer too small");
     memcpy(buf, src.c_str(), src.size() + 1);
@@ -1280,12 +1218,9 @@ up_status up_internal_compile(up_ctx *c, const std::string &src, int rows_per_th
         k->threads = threads;
         if (dyn_smem > 0)
             CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, dyn_smem));
-        if (const char *cv = getenv("UP_SMEM_CARVEOUT"))   // measurement knob: preferred shared-memory carveout (%)
-            CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, atoi(cv)));
         k->dyn_smem = dyn_smem;
         int nb = 0;
         CU_TRY(drv.OccupancyMaxActiveBlocksPerMultiprocessor(&nb, k->fn, threads, (size_t)dyn_smem));
-        if (getenv("UP_PRINT_OCC")) fprintf(stderr, "[libup] %d threads, %d B dynamic smem: %d blocks/SM\n", threads, dyn_smem, nb);
         k->blocks_per_sm = std::max(1, nb);
     }
     *fn_out = k;

@@ -85,31 +85,11 @@ def test_sin_odd_symmetry_on_gpu():
             assert u == ("-" + v if not v.startswith("-") else v[1:])
 
 
-@pytest.mark.parametrize("P,n", [(20, 200), (300, 50), (1400, 6)])
-@pytest.mark.parametrize("pst", [(9, 8), (3, 2), (1, 0)])
-def test_sin_shared_memory_variant(P, n, pst, monkeypatch):
-    """The t-in-shared-memory / S-in-scratch kernel (default for 128 < W <= 200
-    limbs, forced here with UP_SIN_SMEM) against the oracle, incl. scales whose
-    constant shift is a left shift (s = 2) or absent (s = 0)."""
-    monkeypatch.setenv("UP_SIN_SMEM", "1")
-    p, s = pst
-    mag, neg = synth.uniform_decimal(n, p, 5, 4)
-    c = G.ctx()
-    x = c.column_from_host_bin(p, s, mag, neg)
-    out = c.sin_taylor(x, P)
-    c.check()
-    assert c.column_to_strings(out) == oracle.sin_rows(oracle.Column(p, s, mag, neg), P)
-    from paper_conf_icde_lixylz24_b200 import up
-    res = c.sin_taylor_sum(x, P)
-    c.check()
-    assert up.result_to_string(res, P) == oracle.sin_sum(oracle.Column(p, s, mag, neg), P, threads=8)
-
-
 @pytest.mark.parametrize("P,n", [(8, 100), (20, 200), (300, 50), (1000, 12), (1700, 4)])
 @pytest.mark.parametrize("pst", [(9, 8), (8, 7), (3, 2), (1, 0)])
 def test_sin_register_sum_variant(P, n, pst):
     """The default kernel for W <= 200 limbs (t in shared memory, S in
-    registers, chained word divisions; UP_SIN_V2 unset) against the oracle:
+    registers, one 3-by-2 division pass per term) against the oracle:
     scales whose constant shift is a right shift (s = 8, 7), a left shift
     (s = 2) or absent with no constant divisor (s = 0)."""
     p, s = pst
@@ -123,18 +103,6 @@ def test_sin_register_sum_variant(P, n, pst):
     res = c.sin_taylor_sum(x, P)
     c.check()
     assert up.result_to_string(res, P) == oracle.sin_sum(oracle.Column(p, s, mag, neg), P, threads=8)
-
-
-@pytest.mark.parametrize("P", [100, 1000])
-def test_sin_v2_kernels_still_exact(P, monkeypatch):
-    """The previous one-row-per-thread kernels (UP_SIN_V2: t in registers) stay exact."""
-    monkeypatch.setenv("UP_SIN_V2", "1")
-    mag, neg = synth.uniform_decimal(40, 9, 5, 4)
-    c = G.ctx()
-    x = c.column_from_host_bin(9, 8, mag, neg)
-    out = c.sin_taylor(x, P)
-    c.check()
-    assert c.column_to_strings(out) == oracle.sin_rows(oracle.Column(9, 8, mag, neg), P)
 
 
 @pytest.mark.parametrize("lanes", [1, 2, 8, 32])

@@ -73,18 +73,16 @@ def test_wide_edge_values_and_flags():
     ("-c1*c2 + c3*c1 - c2", [(150, 10), (150, 10), (140, 10)], ()),
     ("c1*c2 - c3/c4", [(1000, 100)] * 4, (3,)),
 ])
-@pytest.mark.parametrize("radix", ["tc", "r28", "r32"])
+@pytest.mark.parametrize("radix", ["tc", "r32"])
 def test_split_sum_matches_unsplit_and_oracle(expr, types, lead, radix, monkeypatch):
     """Row-contraction SUM (products as carry-save column sums over rows, signs
     by correction terms) + fused rest kernel + combine == oracle == UP_NO_SPLIT,
     for the tensor-core contraction (default, contract_tc.cu) and the CUDA-core
-    ones (UP_NO_TC: 32-bit, radix-2^28 with UP_CONTRACT28)."""
+    one (UP_NO_TC, also taken beyond 2^31 rows per call)."""
     n = 300 if types[0][0] >= 1000 else 2000
     monkeypatch.setenv("UP_SPLIT", "1")
     if radix != "tc":
         monkeypatch.setenv("UP_NO_TC", "1")
-    if radix == "r28":
-        monkeypatch.setenv("UP_CONTRACT28", "1")
     host = G.gen_cols(n, types, config=3, nonzero_lead_cols=lead, seed=11)
     want, P, S = oracle.eval_sum(expr, G.to_oracle(host, types), threads=8)
     from paper_conf_icde_lixylz24_b200 import up
@@ -101,16 +99,13 @@ def test_split_sum_matches_unsplit_and_oracle(expr, types, lead, radix, monkeypa
 
 
 @pytest.mark.parametrize("p", [200, 1000])
-@pytest.mark.parametrize("radix", ["tc", "r28", "r32"])
+@pytest.mark.parametrize("radix", ["tc", "r32"])
 def test_split_contraction_extreme_values(p, radix, monkeypatch):
-    """All-nines magnitudes (every 28-bit digit near 2^28 - 1, the column-sum
-    bound) with mixed signs over many rows per thread: SUM(c1*c2) by the
-    row contraction (tensor cores, both CUDA-core radices) == exact Python value."""
+    """All-nines magnitudes with mixed signs over many rows per thread:
+    SUM(c1*c2) by the row contraction (tensor cores, CUDA cores) == exact Python value."""
     monkeypatch.setenv("UP_SPLIT", "1")
     if radix != "tc":
         monkeypatch.setenv("UP_NO_TC", "1")
-    if radix == "r28":
-        monkeypatch.setenv("UP_CONTRACT28", "1")
     import numpy as np
     from paper_conf_icde_lixylz24_b200 import up
     n = 5000 if p == 200 else 600
