@@ -45,13 +45,13 @@ namespace {
 
 // bank-conflict-minimising padded row stride (words) for lanes (r, b) that
 // touch word (base - DELTA b) of row r; elt = 1 (u32) or 2 (u64 words)
-int pick_stride(int R, int G, int DELTA, int elt) {
+int pick_stride(int R, int G, int DELTA, int elt, int RPL) {
     int best = R, bestc = 1 << 30;
     for (int rs = R; rs < R + 64; ++rs) {
         int cnt[32] = {0};
-        for (int b = 0; b < G; ++b)
-            for (int r = 0; r < R; ++r) {
-                const long long idx = (long long)(1000 - DELTA * b) * rs + r;
+        for (int b = 0; b < G; ++b)              // one access instruction: row slots g RPL + q, q fixed
+            for (int g = 0; g < 32 / G; ++g) {
+                const long long idx = (long long)(1000 - DELTA * b) * rs + g * RPL;
                 for (int e = 0; e < elt; ++e) cnt[(idx * elt + e) & 31]++;
             }
         int mx = 0;
@@ -116,51 +116,66 @@ __device__ __forceinline__ u32 s_digit(int rr, int jo) {
 }
 __device__ __forceinline__ long long s_top(int rr) { return (long long)Ssm[(WS - 1) * RSS + rr] >> CSC; }
 
-// lanes: rr = row slot of this warp (R = 32 / G rows), b = term index in the band
+// lanes: g = lane / G owns the RPL row slots rr = g RPL + q of this warp
+// (R = RPL 32 / G rows), b = lane % G is the term index in the band; the RPL
+// rows of a lane run the same term (same D_k, o_k, drop, mask) as independent
+// remainder chains interleaved in one instruction stream
 extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
     u32 *const Ysm = YSM;
     const int lane = threadIdx.x;
-    const int rr = lane / G, b = lane % G;
+    const int gl = lane / G, b = lane % G;
+    const int rr0 = gl * RPL;
     const unsigned FULL = 0xFFFFFFFFu;
     u32 fl = 0;
-    for (int l = b; l < WS; l += G) Ssm[l * RSS + rr] = 0ull;
+#pragma unroll
+    for (int q = 0; q < RPL; ++q)
+        for (int l = b; l < WS; l += G) Ssm[l * RSS + rr0 + q] = 0ull;
     int since_norm = 0;
-    u32 acc_neg = 0u;     // SUM: the row slot's accumulator currently holds -(sum)
+    u32 acc_neg[RPL];     // SUM: the row slot's accumulator currently holds -(sum)
+#pragma unroll
+    for (int q = 0; q < RPL; ++q) acc_neg[q] = 0u;
     const long long n = P.n;
     const long long groups = (n + R - 1) / R;
     for (long long grp = blockIdx.x; grp < groups; grp += gridDim.x) {
-        const long long row = grp * R + rr;
-        const bool valid = row < n;
-        const u32 xv = valid ? __ldcs(P.col[0] + row) : 0u;
-        const u32 ng = xv >> 31;
-        const u32 mx = ng ? 0u - xv : xv;
-        const u64 X2 = (u64)mx * mx;
-        const u32 x0 = (u32)X2, x1 = (u32)(X2 >> 32);
-        // ---- Y_1 = |m| 10^(P-s) (slot l = digit l), lane b == 0 of the row
+        u32 ng[RPL], x0[RPL], x1[RPL];
+        bool valid[RPL];
+        long long row[RPL];
         int top = -1;
-        if (b == 0) {
-            u64 c = 0;
-            for (int l = 0; l < W; ++l) {
-                const u64 q = mulw(POW10PS[l], mx) + c;
-                const u32 v = (u32)q;
-                Ysm[l * RSY + rr] = v;
-                c = q >> 32;
-                if (v) top = l;
-            }
-            for (int l = W; l < WY; ++l) Ysm[l * RSY + rr] = 0u;
-#if !SUM
-            for (int l = 0; l < WS; ++l) Ssm[l * RSS + rr] = 0ull;
-#endif
-        }
+#pragma unroll
+        for (int q = 0; q < RPL; ++q) {
+            const int rr = rr0 + q;
+            row[q] = grp * R + rr;
+            valid[q] = row[q] < n;
+            const u32 xv = valid[q] ? __ldcs(P.col[0] + row[q]) : 0u;
+            ng[q] = xv >> 31;
+            const u32 mx = ng[q] ? 0u - xv : xv;
+            const u64 X2 = (u64)mx * mx;
+            x0[q] = (u32)X2;
+            x1[q] = (u32)(X2 >> 32);
+            // ---- Y_1 = |m| 10^(P-s) (slot l = digit l), lane b == 0 of the row group
+            if (b == 0) {
+                u64 c = 0;
+                for (int l = 0; l < W; ++l) {
+                    const u64 t = mulw(POW10PS[l], mx) + c;
+                    const u32 v = (u32)t;
+                    Ysm[l * RSY + rr] = v;
+                    c = t >> 32;
+                    if (v && l > top) top = l;
+                }
+                for (int l = W; l < WY; ++l) Ysm[l * RSY + rr] = 0u;
 #if SUM
-        // sum of sign(m) S over rows: the slot accumulates with the sign of the
-        // current row; negate it in place when the sign changes
-        if (b == 0 && ng != acc_neg) {
-            for (int l = 0; l < WS; ++l) Ssm[l * RSS + rr] = 0ull - Ssm[l * RSS + rr];
-            acc_neg = ng;
-        }
+                // sum of sign(m) S over rows: the slot accumulates with the sign of the
+                // current row; negate it in place when the sign changes
+                if (ng[q] != acc_neg[q]) {
+                    for (int l = 0; l < WS; ++l) Ssm[l * RSS + rr] = 0ull - Ssm[l * RSS + rr];
+                    acc_neg[q] = ng[q];
+                }
+#else
+                for (int l = 0; l < WS; ++l) Ssm[l * RSS + rr] = 0ull;
 #endif
-        top = __shfl_sync(FULL, top, rr * G);
+            }
+        }
+        top = __shfl_sync(FULL, top, gl * G);
         __syncwarp();
         int J0 = (int)__reduce_max_sync(FULL, (unsigned)(top + 1)) - 1 + 3 + SDMAX;   // top + 3 + sd
         bool live = __any_sync(FULL, top >= 0);
@@ -179,17 +194,9 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
             const u32 onew = o2 & 31u;
             const u32 mask = onew ? ~((1u << onew) - 1u) : 0xFFFFFFFFu;
             const u32 esh = CSC - o;                      // S addend = Y_k digit << esh
-            const bool negt = (k & 1u) == 0u;                  // (-1)^(k-1)
-            u32 r1 = 0u, r0 = 0u, qprev = 0u;
-            u32 p0a = 0u, p0b = 0u, p1a = 0u;      // p0 of y loaded 1 / 2 steps ago, p1 of 1 step ago
-            u32 Alo = 0u;                           // low word of the previous step's A
+            const bool negt = (k & 1u) == 0u;             // (-1)^(k-1)
             const int jb = J0 + DELTA * b, jtop = J0 + b;
             const int steps = DELTA * (G - 1) + J0 + 1;
-            // running shared-window byte addresses of this step's load / store slots
-            const u32 ybase = (u32)__cvta_generic_to_shared(Ysm), sbase = (u32)__cvta_generic_to_shared(Ssm);
-            u32 yl = ybase + 4u * (u32)((jb - 3 - sd) * RSY + rr);
-            u32 yw = ybase + 4u * (u32)((jb - drop) * RSY + rr);
-            u32 sl = sbase + 8u * (u32)((jb - 3 - sd) * RSS + rr);
             const int jld = 3 + sd;
 #if NEGSH0
             // negative terms have esh = 0: add ~y (= 2^32 - 1 - y) per loaded slot, then
@@ -198,8 +205,11 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
             if (negt) {
                 const int nl = jtop - 2 - sd;
                 if (nl > 0) {
-                    atomicAdd(&Ssm[nl * RSS + rr], ~0ull);
-                    atomicAdd(&Ssm[rr], 1ull);
+#pragma unroll
+                    for (int q = 0; q < RPL; ++q) {
+                        atomicAdd(&Ssm[nl * RSS + rr0 + q], ~0ull);
+                        atomicAdd(&Ssm[rr0 + q], 1ull);
+                    }
                 }
             }
             __syncwarp();
@@ -207,72 +217,90 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
             const u64 smsk = negt ? ~0ull : 0ull;
 #endif
             const u32 nd1 = 0u - d1;
+            u32 r1[RPL], r0[RPL], qprev[RPL], p0a[RPL], p0b[RPL], p1a[RPL], Alo[RPL], ynext[RPL];
+            // running shared-window byte addresses of row rr0's load / store slots (row q: + 4q / 8q)
+            const u32 ybase = (u32)__cvta_generic_to_shared(Ysm), sbase = (u32)__cvta_generic_to_shared(Ssm);
+            u32 yl = ybase + 4u * (u32)((jb - 3 - sd) * RSY + rr0);
+            u32 yw = ybase + 4u * (u32)((jb - drop) * RSY + rr0);
+            u32 sl = sbase + 8u * (u32)((jb - 3 - sd) * RSS + rr0);
             // software pipeline: the digit step tau + 1 consumes was written at step <= tau - 1
             // (DELTA >= 6 + sd), so it is loaded one step ahead, off the remainder chain
-            u32 ynext = lds32p((unsigned)jb <= (unsigned)jtop && jb >= jld, yl);
-#pragma unroll 2
+            const bool ld0 = (unsigned)jb <= (unsigned)jtop && jb >= jld;
+#pragma unroll
+            for (int q = 0; q < RPL; ++q) {
+                r1[q] = r0[q] = qprev[q] = p0a[q] = p0b[q] = p1a[q] = Alo[q] = 0u;
+                ynext[q] = lds32p(ld0, yl + 4u * q);
+            }
+#pragma unroll 1
             for (int tau = 0; tau < steps; ++tau) {
                 const int j = jb - tau;
                 const bool act = (unsigned)j <= (unsigned)jtop;
                 const bool ld = act && j >= jld;
-                const u32 y = ynext;
-                ynext = lds32p((unsigned)(j - 1) <= (unsigned)jtop && j - 1 >= jld, yl - 4u * RSY);
-                {   // running sum: S 2^c += (-1)^(k-1) Y_k 2^(c - o_k)   (y = 0: no-op)
+                const bool ldn = (unsigned)(j - 1) <= (unsigned)jtop && j - 1 >= jld;
+                const bool st = act && j >= drop;
+                const u32 qm = j == drop ? mask : 0xFFFFFFFFu;
+#pragma unroll
+                for (int q = 0; q < RPL; ++q) {
+                    const u32 y = ynext[q];
+                    ynext[q] = lds32p(ldn, yl - 4u * RSY + 4u * q);
+                    {   // running sum: S 2^c += (-1)^(k-1) Y_k 2^(c - o_k)   (y = 0: no-op)
 #if NEGSH0
-                    const u64 a = ((u64)y << esh) ^ xm;
+                        const u64 a = ((u64)y << esh) ^ xm;
 #else
-                    const u64 a = (((u64)y << esh) ^ smsk) - smsk;
+                        const u64 a = (((u64)y << esh) ^ smsk) - smsk;
 #endif
+                        const u32 sq = sl + 8u * q;
 #if SPLIT
-                    const u64 s0 = lds64p(ld, sl), s1 = lds64p(ld, sl + 8u * RSS);
-                    const long long sa = (long long)a;
-                    sts64p(ld, sl, s0 + (u64)(u32)(u64)sa);
-                    sts64p(ld, sl + 8u * RSS, s1 + (u64)(sa >> 32));
+                        const u64 s0 = lds64p(ld, sq), s1 = lds64p(ld, sq + 8u * RSS);
+                        const long long sa = (long long)a;
+                        sts64p(ld, sq, s0 + (u64)(u32)(u64)sa);
+                        sts64p(ld, sq + 8u * RSS, s1 + (u64)(sa >> 32));
 #else
-                    sts64p(ld, sl, lds64p(ld, sl) + a);
+                        sts64p(ld, sq, lds64p(ld, sq) + a);
 #endif
-                }
-                // product digit stream: y X2 = p0 + p1 B + p2 B^2
-                const u64 pa = mulw(y, x0);
-                const u64 pb = mulw(y, x1);
-                u32 p1, p2;
-                asm("add.cc.u32 %0, %2, %3; addc.u32 %1, %4, 0;" : "=r"(p1), "=r"(p2)
-                    : "r"((u32)pb), "r"((u32)(pa >> 32)), "r"((u32)(pb >> 32)));
-                const u32 p0 = (u32)pa;
-                // A at the new position = p0(2 ago) + p1(1 ago) + p2(now)  (< 3B)
-                const u64 A = (u64)p0b + p1a + p2;
-                // V digit: lo32(Aprev << sb) + (A >> (32 - sb)); its carry goes into R
-                const u64 vs = (u64)(Alo << sb) + (A >> (32u - sb));
-                const u32 u0 = (u32)vs;
-                u64 T = (((u64)r1 << 32) | r0) + (vs >> 32);
-                if (__builtin_expect(T >= Dn, 0)) {   // quotient digit >= B (p ~ 2^-63): +1 into the digit emitted last step
-                    T -= Dn;
-                    if (act && j + 1 <= jtop) {
-                        const u32 pv = qprev + 1u;
-                        if (pv == 0u) fl |= F_INVAL;   // second-order ripple (p ~ 2^-95): flagged, never silent
-                        sts32p(j + 1 >= drop, yw + 4u * RSY, j + 1 == drop ? (pv & mask) : pv);
                     }
+                    // product digit stream: y X2 = p0 + p1 B + p2 B^2
+                    const u64 pa = mulw(y, x0[q]);
+                    const u64 pb = mulw(y, x1[q]);
+                    u32 p1, p2;
+                    asm("add.cc.u32 %0, %2, %3; addc.u32 %1, %4, 0;" : "=r"(p1), "=r"(p2)
+                        : "r"((u32)pb), "r"((u32)(pa >> 32)), "r"((u32)(pb >> 32)));
+                    const u32 p0 = (u32)pa;
+                    // A at the new position = p0(2 ago) + p1(1 ago) + p2(now)  (< 3B)
+                    const u64 A = (u64)p0b[q] + p1a[q] + p2;
+                    // V digit: lo32(Aprev << sb) + (A >> (32 - sb)); its carry goes into R
+                    const u64 vs = (u64)(Alo[q] << sb) + (A >> (32u - sb));
+                    const u32 u0 = (u32)vs;
+                    u64 T = (((u64)r1[q] << 32) | r0[q]) + (vs >> 32);
+                    if (__builtin_expect(T >= Dn, 0)) {   // quotient digit >= B (p ~ 2^-63): +1 into the digit emitted last step
+                        T -= Dn;
+                        if (act && j + 1 <= jtop) {
+                            const u32 pv = qprev[q] + 1u;
+                            if (pv == 0u) fl |= F_INVAL;   // second-order ripple (p ~ 2^-95): flagged, never silent
+                            sts32p(j + 1 >= drop, yw + 4u * RSY + 4u * q, j + 1 == drop ? (pv & mask) : pv);
+                        }
+                    }
+                    // Moller-Granlund 3-by-2 step (T:u0) / Dn, T < Dn
+                    u32 qd;
+                    {
+                        const u32 u2 = (u32)(T >> 32), u1 = (u32)T;
+                        const u64 qq = mulw(v, u2) + T;
+                        u32 q1 = (u32)(qq >> 32);
+                        const u32 q0 = (u32)qq;
+                        const u32 rh = u1 + q1 * nd1;
+                        u64 rm = ((((u64)rh) << 32) | u0) - mulw(d0, q1) - Dn;
+                        q1 += 1u;
+                        if ((u32)(rm >> 32) >= q0) { q1 -= 1u; rm += Dn; }
+                        if (__builtin_expect(rm >= Dn, 0)) { q1 += 1u; rm -= Dn; }
+                        r1[q] = (u32)(rm >> 32);
+                        r0[q] = (u32)rm;
+                        qd = q1;
+                    }
+                    sts32p(st, yw + 4u * q, qd & qm);
+                    qprev[q] = qd;
+                    p0b[q] = p0a[q]; p0a[q] = p0; p1a[q] = p1;
+                    Alo[q] = (u32)A;
                 }
-                // Moller-Granlund 3-by-2 step (T:u0) / Dn, T < Dn
-                u32 q;
-                {
-                    const u32 u2 = (u32)(T >> 32), u1 = (u32)T;
-                    const u64 qq = mulw(v, u2) + T;
-                    u32 q1 = (u32)(qq >> 32);
-                    const u32 q0 = (u32)qq;
-                    const u32 rh = u1 + q1 * nd1;
-                    u64 rm = ((((u64)rh) << 32) | u0) - mulw(d0, q1) - Dn;
-                    q1 += 1u;
-                    if ((u32)(rm >> 32) >= q0) { q1 -= 1u; rm += Dn; }
-                    if (__builtin_expect(rm >= Dn, 0)) { q1 += 1u; rm -= Dn; }
-                    r1 = (u32)(rm >> 32);
-                    r0 = (u32)rm;
-                    q = q1;
-                }
-                sts32p(act && j >= drop, yw, q & (j == drop ? mask : 0xFFFFFFFFu));
-                qprev = q;
-                p0b = p0a; p0a = p0; p1a = p1;
-                Alo = (u32)A;
                 yl -= 4u * RSY; yw -= 4u * RSY; sl -= 8u * RSS;
                 __syncwarp();
             }
@@ -283,12 +311,16 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
             int tp = -1;
             if (b == 0) {
                 const u32 ol = (TWO_S * (kbase - 2u)) & 31u;
-                tp = J0 + G - 1 - (int)((ol + TWO_S) >> 5);
-                if (tp > WY - 1) tp = WY - 1;
-                while (tp >= 0 && Ysm[tp * RSY + rr] == 0u) --tp;
-                for (int l = tp + 1; l <= tp + SDMAX + 3 && l < WY; ++l) Ysm[l * RSY + rr] = 0u;
+                const int t0 = min(J0 + G - 1 - (int)((ol + TWO_S) >> 5), WY - 1);
+#pragma unroll
+                for (int q = 0; q < RPL; ++q) {
+                    int t = t0;
+                    while (t >= 0 && Ysm[t * RSY + rr0 + q] == 0u) --t;
+                    for (int l = t + 1; l <= t + SDMAX + 3 && l < WY; ++l) Ysm[l * RSY + rr0 + q] = 0u;
+                    tp = max(tp, t);
+                }
             }
-            tp = __shfl_sync(FULL, tp, rr * G);
+            tp = __shfl_sync(FULL, tp, gl * G);
             live = __any_sync(FULL, tp >= 0);
             J0 = (int)__reduce_max_sync(FULL, (unsigned)(tp + 1)) - 1 + 3 + SDMAX;
             if (kbase > KT + G) { fl |= F_INVAL; break; }
@@ -296,17 +328,26 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
         }
         // ---- row end
 #if SUM
-        if (++since_norm >= NR) { since_norm = 0; if (b == 0) s_normalize(rr); }
+        if (++since_norm >= NR) {
+            since_norm = 0;
+            if (b == 0)
+#pragma unroll
+                for (int q = 0; q < RPL; ++q) s_normalize(rr0 + q);
+        }
 #else
         if (b == 0) {
-            s_normalize(rr);
-            // out = sign(m) (S 2^c >> c), two's complement, LO limbs
-            const u32 msk = 0u - ng;
-            u32 cy = ng;
-            for (int jo = 0; jo < LO; ++jo) {
-                const u64 t = (u64)(s_digit(rr, jo) ^ msk) + cy;
-                cy = (u32)(t >> 32);
-                if (valid) P.out[(long long)jo * P.ld_out + row] = (u32)t;
+#pragma unroll
+            for (int q = 0; q < RPL; ++q) {
+                const int rr = rr0 + q;
+                s_normalize(rr);
+                // out = sign(m) (S 2^c >> c), two's complement, LO limbs
+                const u32 msk = 0u - ng[q];
+                u32 cy = ng[q];
+                for (int jo = 0; jo < LO; ++jo) {
+                    const u64 t = (u64)(s_digit(rr, jo) ^ msk) + cy;
+                    cy = (u32)(t >> 32);
+                    if (valid[q]) P.out[(long long)jo * P.ld_out + row[q]] = (u32)t;
+                }
             }
         }
 #endif
@@ -314,18 +355,22 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
     }
     if (fl) atomicOr(P.flags, fl);
 #if SUM
-    // commit this row slot's S (signed, x 2^c) into the pos / neg workspace
+    // commit this lane's row slots' S (signed, x 2^c) into the pos / neg workspace
     if (b == 0) {
-        if (acc_neg)
-            for (int l = 0; l < WS; ++l) Ssm[l * RSS + rr] = 0ull - Ssm[l * RSS + rr];
-        s_normalize(rr);
-        for (int jo = 0; jo < WS - 1; ++jo) {
-            const u32 dgt = s_digit(rr, jo);
-            if (dgt) atomicAdd(&P.ws[jo], (u64)dgt);
+#pragma unroll
+        for (int q = 0; q < RPL; ++q) {
+            const int rr = rr0 + q;
+            if (acc_neg[q])
+                for (int l = 0; l < WS; ++l) Ssm[l * RSS + rr] = 0ull - Ssm[l * RSS + rr];
+            s_normalize(rr);
+            for (int jo = 0; jo < WS - 1; ++jo) {
+                const u32 dgt = s_digit(rr, jo);
+                if (dgt) atomicAdd(&P.ws[jo], (u64)dgt);
+            }
+            const long long tv = s_top(rr);
+            if (tv > 0) atomicAdd(&P.ws[WS - 1], (u64)tv);
+            if (tv < 0) atomicAdd(&P.ws[WS + WS - 1], (u64)(-tv));
         }
-        const long long tv = s_top(rr);
-        if (tv > 0) atomicAdd(&P.ws[WS - 1], (u64)tv);
-        if (tv < 0) atomicAdd(&P.ws[WS + WS - 1], (u64)(-tv));
     }
     __threadfence();
     __syncwarp();
@@ -358,7 +403,7 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
 }  // namespace
 
 std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum, int G_req, SinBandInfo &info,
-                                std::string &err) {
+                                std::string &err, int rpl_req) {
     if (p > 9 || s > p || s > P || p - s > 1 || 2 * s >= 32) { err = "band sine: unsupported type"; return ""; }
     const int W = limbs_for_precision(P + 23) + 2;
     // number of terms: t_(k+1) <= t_k x^2 / ((2k)(2k+1)), |x| < 10^(p-s)
@@ -373,7 +418,9 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
     // lanes per row (measured, profiles/r02_s2-s3): P = 5000 (W = 520) G = 16, P = 20000 G = 32
     if (G <= 0) G = W <= 160 ? 4 : W <= 700 ? 16 : 32;
     if (G != 1 && G != 2 && G != 4 && G != 8 && G != 16 && G != 32) { err = "band sine: G must divide 32"; return ""; }
-    const int R = 32 / G;
+    const int RPL = rpl_req > 0 ? rpl_req : 2;   // rows per lane: independent chains per instruction stream
+    if (RPL != 1 && RPL != 2 && RPL != 4) { err = "band sine: rows per lane must be 1, 2 or 4"; return ""; }
+    const int R = RPL * 32 / G;
     const int KT = kmax + G + 2;
     // D_k table (normalised), sh split into (sd, sb)
     std::vector<uint32_t> tab;
@@ -402,7 +449,7 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
     int NR = 1;
     if (!split) NR = (int)std::max(1.0, std::floor(std::pow(2.0, 61.0 - per_row)));
     else NR = (int)std::max(1.0, std::floor(std::pow(2.0, 61.0 - (std::log2((double)kmax + G) + 33))));
-    const int RSY = pick_stride(R, G, DELTA, 1), RSS = pick_stride(R, G, DELTA, 2);
+    const int RSY = pick_stride(R, G, DELTA, 1, RPL), RSS = pick_stride(R, G, DELTA, 2, RPL);
     // negative (even-k) terms have o_k = c for every even k (s = 8: o = 16; s = 0: o = 0)
     bool negsh0 = true;
     for (int kk = 2; kk <= 64; kk += 2) negsh0 = negsh0 && (((2 * s * (kk - 1)) & 31) == csc);
@@ -420,7 +467,7 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
       << " G=" << G << " DELTA=" << DELTA << " KT=" << KT << (sum ? " SUM" : " eval") << "\n";
     k << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n";
     k << "#define W " << W << "\n#define WY " << WY << "\n#define WS " << WS << "\n#define G " << G << "\n#define R "
-      << R << "\n#define DELTA " << DELTA << "\n#define SDMAX " << sdmax << "\n#define KT " << KT << "\n#define TWO_S "
+      << R << "\n#define RPL " << RPL << "\n#define DELTA " << DELTA << "\n#define SDMAX " << sdmax << "\n#define KT " << KT << "\n#define TWO_S "
       << 2 * s << "u\n#define CSC " << csc << "\n#define SPLIT " << (split ? 1 : 0) << "\n#define NR " << NR
       << "\n#define NEGSH0 " << (negsh0 ? 1 : 0) << "\n#define RSY " << RSY << "\n#define RSS " << RSS << "\n#define SUM " << (sum ? 1 : 0) << "\n#define LO "
       << Lout << "\n#define LA " << LA << "\n";
