@@ -237,11 +237,12 @@ up_status up_filter(up_ctx *ctx, const char *lhs, const char *op, const char *rh
  * increasing with the key.  *n_groups (host) = number of groups; the call
  * synchronises the stream to read it.  d_first (device int64, optional,
  * n entries): d_first[g] = the smallest row index of group g, for
- * g < *n_groups.  Implementation: stable LSD radix sort (CUB
- * DeviceRadixSort, one pass per 32-bit limb, least significant key column
+ * g < *n_groups.  Implementation (groupby.cu, hand-written): stable LSD
+ * radix sort of (key limb, row) pairs, 8-bit digits (tile histograms, a scan
+ * of the digit-major counts, a stable scatter), least significant key column
  * and limb first, the top limb's sign bit flipped so two's complement orders
- * as signed; excluded rows sorted last), an adjacent-difference pass over all
- * limbs, a prefix sum and a scatter.  Scratch: the ctx's persistent scratch
+ * as signed; excluded rows sorted last; then an adjacent-difference pass over
+ * all limbs, a prefix sum and a scatter.  Scratch: the ctx's persistent scratch
  * buffer (24 bytes per row + sort temporaries), grown on demand (growing it
  * synchronises the device); the call holds the ctx lock throughout.
  */
