@@ -418,7 +418,10 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
     // lanes per row (measured, profiles/r02_s2-s3): P = 5000 (W = 520) G = 16, P = 20000 G = 32
     if (G <= 0) G = W <= 160 ? 4 : W <= 700 ? 16 : 32;
     if (G != 1 && G != 2 && G != 4 && G != 8 && G != 16 && G != 32) { err = "band sine: G must divide 32"; return ""; }
-    const int RPL = rpl_req > 0 ? rpl_req : 2;   // rows per lane: independent chains per instruction stream
+    // rows per lane: independent remainder chains per instruction stream; measured
+    // (profiles/r02_s5) RPL = 2 / 4 halve the resident warps (shared memory per
+    // row) for no ILP gain: P = 5000 9.3e5 (RPL 1) vs 6.5e5 (2) vs 3.5e5 (4) rows/s
+    const int RPL = rpl_req > 0 ? rpl_req : 1;
     if (RPL != 1 && RPL != 2 && RPL != 4) { err = "band sine: rows per lane must be 1, 2 or 4"; return ""; }
     const int R = RPL * 32 / G;
     const int KT = kmax + G + 2;
