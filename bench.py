@@ -207,9 +207,60 @@ class ExprWorkload(Workload):
              "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks
              else "fallback 6.65 TB/s"}
         if self.cfg["types"][0][0] >= 100:
-            r["note"] = ("step = tensor-core row contraction SUM(c1*c2) (u8 digits, s32 TMEM accumulators) "
-                         "+ fused per-thread rest (top-limb division) + exact combine")
+            r = self._split_roofline(kernel_ms, peaks)
         return r
+
+    def _time(self, fn, reps=5):
+        import torch
+        st = torch.cuda.current_stream()
+        fn()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(st)
+        for _ in range(reps):
+            fn()
+        b.record(st)
+        torch.cuda.synchronize()
+        return a.elapsed_time(b) / reps
+
+    def _split_roofline(self, step_ms, peaks):
+        """cfg3 with the tensor-core split: per-kernel fractions, each on what
+        that kernel does.  SUM(c1*c2) alone launches the tcgen05 contraction
+        (it reads c1, c2 whole: 2 x 4L B/row, HBM roofline); SUM(c3/c4) alone
+        launches the fused rest kernel (top-limb division: reads a window of
+        c3/c4's top limbs, integer roofline on the SURVEY's division count).
+        The line's roofline is the dominant (contraction) kernel's."""
+        import torch
+        from paper_conf_icde_lixylz24_b200 import up
+        p, s = self.cfg["types"][0]
+        L = up.limbs(p)
+        c1, c2, c3, c4 = self.cols
+        out = torch.empty(self.LA, dtype=torch.int32, device="cuda")
+        t_tc = self._time(lambda: self.ctx.sum_expr("c1*c2", [c1, c2], self.n_global, out=out))
+        t_rest = self._time(lambda: self.ctx.sum_expr("c1/c2", [c3, c4], self.n_global, out=out))
+        peak = peaks.get("hbm_gbs", 6650.0)
+        tc_bytes = 2 * 4 * L * self.rows
+        ach = tc_bytes / (t_tc / 1e3) / 1e9
+        mag = lambda k: max(1, (10 ** k).bit_length() // 32 + 1)   # noqa: E731
+        nu = mag(p + s + 4)
+        div_products = L * mag(s + 4) + (nu - L + 1) * L
+        pk, src = _product_peak()
+        rest_ach = div_products * self.rows / (t_rest / 1e3)
+        return {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
+                "kernel_ms": round(t_tc, 5), "alg_bytes_per_launch": tc_bytes,
+                "alg_unit": f"contraction kernel: c1, c2 limb planes {2 * 4 * L} B/row x {self.rows} rows",
+                "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s",
+                "kernels": [
+                    {"kernel": "k_contract_tc (SUM(c1*c2), tcgen05 kind::i8)", "ms": round(t_tc, 5), "bound": "hbm",
+                     "alg_bytes": tc_bytes, "achieved_gbs": round(ach, 1), "frac": round(ach / peak, 4)},
+                    {"kernel": "upk rest (SUM(-c3/c4), top-limb division)", "ms": round(t_rest, 5), "bound": "alu",
+                     "alg_products": div_products * self.rows,
+                     "alg_unit": f"{div_products} limb products/row (SURVEY 8d division count; the kernel decides "
+                                 "most quotients from the top limbs and does fewer)",
+                     "achieved_T_products_s": round(rest_ach / 1e12, 4), "frac": round(rest_ach / pk, 4),
+                     "peak_source": src}],
+                "step_ms": round(step_ms, 5),
+                "note": "step = contraction + rest + exact combine, back to back on one stream"}
 
     def alg_products_per_row(self):
         """limb products of c1*c2 - c3/c4 = x (L*L) + / prescale

@@ -194,6 +194,21 @@ up_status up_group_aggregate(up_ctx *ctx, int32_t n_aggs, const int32_t *kinds, 
                              int64_t n_global, uint32_t *d_out, uint64_t *d_counts, void *stream);
 
 /*
+ * Per-operator kernels with TPI threads per instance (the
+ * paper's multi-threading arithmetic, Sec. III-E1, Fig. 13):
+ * out = a <op> b per row, op "+" "-" "*" "/", with the values, types and
+ * flags of up_eval_expr("c1<op>c2").  A group of tpi lanes
+ * (1, 2, 4, 8, 16, 32) owns each row: + - * run on every tpi; "/" runs one row
+ * per thread (tpi 1) with div_algo 0 = long division (Knuth D, the fused
+ * kernels' method) or 1 = Newton-Raphson reciprocal iteration,
+ * operands up to 64 limbs.  Inputs: limb planes or compact rows (compact rows
+ * are read by the group as in the paper's Listing 3); out: limb planes,
+ * caller-allocated with the expression's type.  One kernel launch.
+ */
+up_status up_eval_tpi(up_ctx *ctx, const char *op, const up_column *a, const up_column *b, int32_t tpi,
+                      int32_t div_algo, up_column *out, void *stream);
+
+/*
  * Multi-rank GROUP BY (NEXT-4 with rows a13/e): every rank runs
  * up_group_aggregate over its rows with each AVG replaced by SUM (the
  * combinable partial state of an average; same n_global on every rank), the
@@ -314,6 +329,8 @@ up_status up_gen_sin_source(int32_t P, int32_t p, int32_t s, int sum, int64_t n_
 up_status up_gen_group_agg_source(int32_t n_aggs, const int32_t *kinds, const char *const *exprs,
                                   const up_column *cols, int ncols, int32_t n_groups, int64_t n_global,
                                   char *buf, size_t len);
+/* Generated up_eval_tpi source for cols[0] <op> cols[1] (types / layouts only). */
+up_status up_gen_tpi_source(const char *op, const up_column *cols, int32_t tpi, int32_t div_algo, char *buf, size_t len);
 /* Generated modexp source for a DECIMAL(base_p,0) base (sum != 0: fused SUM variant). */
 up_status up_gen_modexp_source(const char *exponent, const char *modulus, int32_t base_p, int sum,
                                int64_t n_global, char *buf, size_t len);

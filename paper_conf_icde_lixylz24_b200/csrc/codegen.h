@@ -62,6 +62,12 @@ struct ModexpPlan {
 std::string gen_modexp_kernel(const HBig &N, const HBig &e, const ModexpPlan &plan, bool sum, std::string &err);
 std::string gen_sin_kernel(int P, int p, int s, int Lx, int Lout, int LA, bool sum, int &lanes_per_row, std::string &err,
                            int *smem_per_thread = nullptr, bool *is_v3 = nullptr);
+// per-operator kernels with TPI lanes per row (tpi.cpp, NEXT-3); op: 0 + 1 - 2 * 3 /
+struct TpiInfo {
+    int rows_per_block = 0, dyn_smem = 0;
+};
+std::string gen_tpi_kernel(int op, const ColType &ta, const ColType &tb, const Node *root, int G, bool nr_div,
+                           TpiInfo &info, std::string &err);
 // skewed-band sine (sin_band.cpp): one warp per block, R = 32 / G rows per warp
 struct SinBandInfo {
     int G = 0, rows_per_block = 0, smem = 0, ws_slots = 0, delta = 0, W = 0;

@@ -224,7 +224,7 @@ up_status need_planes(const up_column *col, const char *what) {
     return UP_OK;
 }
 
-const char *kNvrtcOpts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-default-device", "-lineinfo", "-DNDEBUG"};
+const char *kNvrtcOpts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-default-device", "-lineinfo", "-DNDEBUG", "--device-int128"};
 
 // On-disk cubin cache (keyed by FNV-1a of source + options + embedded header):
 // $UP_JIT_CACHE, else <dir of libup.so>/_jitcache.  Purely a compile-time
@@ -1032,6 +1032,51 @@ up_status up_agg_type(const char *expr, int32_t kind, const up_column *cols, int
     return UP_OK;
 }
 
+up_status up_eval_tpi(up_ctx *c, const char *op, const up_column *a, const up_column *b, int32_t tpi, int32_t div_algo,
+                      up_column *out, void *stream) {
+    if (!c || !op || !a || !b || !out) return fail(UP_E_INVAL, "need a ctx, an operator, two columns and out");
+    int o = -1;
+    if (!strcmp(op, "+")) o = 0;
+    if (!strcmp(op, "-")) o = 1;
+    if (!strcmp(op, "*")) o = 2;
+    if (!strcmp(op, "/")) o = 3;
+    if (o < 0) return fail(UP_E_INVAL, "operator must be + - * /");
+    if (div_algo != 0 && div_algo != 1) return fail(UP_E_INVAL, "div_algo must be 0 (long division) or 1 (Newton-Raphson)");
+    const up_column cols[2] = {*a, *b};
+    for (int i = 0; i < 2; ++i)
+        if (up_status s = check_column(&cols[i], "input")) return s;
+    if (a->n != b->n) return fail(UP_E_INVAL, "columns differ in length");
+    if (up_status s = check_column(out, "out")) return s;
+    if (out->layout != UP_LAYOUT_PLANES) return fail(UP_E_UNSUPPORTED, "out must be limb planes");
+    const std::string expr = std::string("c1") + op + "c2";
+    Typed t;
+    if (up_status s = type_expr(expr.c_str(), cols, 2, t)) return s;
+    if (out->p != t.root->p || out->s != t.root->s || out->n != a->n)
+        return fail(UP_E_INVAL, "out must be DECIMAL(%d,%d) with the inputs' rows", t.root->p, t.root->s);
+    if (o == 3 && (t.root->l->L > 64 || t.root->r->L > 64 || t.root->L > 64))
+        return fail(UP_E_UNSUPPORTED, "tpi division: operands up to 64 limbs");
+    std::lock_guard<std::mutex> g(c->mu);
+    std::string key = "tpi|" + expr + "|" + std::to_string(tpi) + "|" + std::to_string(div_algo);
+    for (int i = 0; i < 2; ++i)
+        key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s) + (cols[i].layout ? "c" : "");
+    JitKernel *k = nullptr;
+    std::string err;
+    TpiInfo ti;
+    if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
+            std::string src = gen_tpi_kernel(o, t.types[0], t.types[1], t.root.get(), tpi, div_algo == 1, ti, err);
+            info.threads = 256;
+            info.dyn_smem = ti.dyn_smem;
+            return src; }, &k))
+        return err.empty() ? s : fail(UP_E_UNSUPPORTED, "%s", err.c_str());
+    up_kparams P;
+    fill_cols(P, cols, 2);
+    P.flags = c->d_flags;
+    P.out = out->data;
+    P.ld_out = out->ld;
+    if (P.n == 0) return UP_OK;
+    return launch(c, k, P, P.n * (long long)tpi, (cudaStream_t)stream);
+}
+
 up_status up_group_combine(up_ctx *c, int32_t n_aggs, const int32_t *kinds, const char *const *exprs,
                            const up_column *cols, int ncols, int32_t n_groups, int64_t n_global, const uint32_t *d_parts,
                            int32_t nranks, const uint64_t *d_counts, uint32_t *d_out, uint64_t *d_counts_out,
@@ -1123,6 +1168,22 @@ up_status up_gen_group_agg_source(int32_t n_aggs, const int32_t *kinds, const ch
 }
 
 // ---- diagnostics (no GPU needed): generated source and an NVRTC-only compile
+up_status up_gen_tpi_source(const char *op, const up_column *cols, int32_t tpi, int32_t div_algo, char *buf, size_t len) {
+    if (!op || !cols) return fail(UP_E_INVAL, "null argument");
+    const int o = !strcmp(op, "+") ? 0 : !strcmp(op, "-") ? 1 : !strcmp(op, "*") ? 2 : !strcmp(op, "/") ? 3 : -1;
+    if (o < 0) return fail(UP_E_INVAL, "operator must be + - * /");
+    const std::string expr = std::string("c1") + op + "c2";
+    Typed t;
+    if (up_status s = type_expr(expr.c_str(), cols, 2, t)) return s;
+    TpiInfo ti;
+    std::string err;
+    const std::string src = gen_tpi_kernel(o, t.types[0], t.types[1], t.root.get(), tpi, div_algo == 1, ti, err);
+    if (src.empty()) return fail(UP_E_UNSUPPORTED, "%s", err.c_str());
+    if (src.size() + 1 > len) return fail(UP_E_NOMEM, "buffer too small");
+    memcpy(buf, src.c_str(), src.size() + 1);
+    return UP_OK;
+}
+
 up_status up_gen_source(const char *variant, const char *expr, const up_column *cols, int ncols, int64_t n_global,
                         char *buf, size_t len) {
     if (!variant || !buf) return fail(UP_E_INVAL, "null argument");

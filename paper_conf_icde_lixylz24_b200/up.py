@@ -40,7 +40,8 @@ EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_l
            "up_jit_ms", "up_gen_source", "up_nvrtc_compile", "up_gen_modexp_source", "up_jit_prewarm", "up_gen_sin_source", "up_compact_bytes",
            "up_column_from_host_compact", "up_column_from_device_compact", "up_column_to_host_compact",
            "up_expr_optimized", "up_gen_contract_source", "up_agg_type", "up_group_aggregate",
-           "up_gen_group_agg_source", "up_filter", "up_group_ids", "up_group_combine"]
+           "up_gen_group_agg_source", "up_filter", "up_group_ids", "up_group_combine", "up_eval_tpi",
+           "up_gen_tpi_source"]
 
 AGG = {"SUM": 0, "MIN": 1, "MAX": 2, "AVG": 3}
 
@@ -100,6 +101,8 @@ def lib():
                                           c.c_int64, c.c_char_p, c.c_size_t]
     L.up_filter.argtypes = [P, c.c_char_p, c.c_char_p, c.c_char_p, PC, c.c_int, P, P]
     L.up_group_ids.argtypes = [P, PC, c.c_int, P, c.POINTER(c.c_int64), P, P]
+    L.up_eval_tpi.argtypes = [P, c.c_char_p, PC, PC, c.c_int32, c.c_int32, PC, P]
+    L.up_gen_tpi_source.argtypes = [c.c_char_p, PC, c.c_int32, c.c_int32, c.c_char_p, c.c_size_t]
     L.up_group_combine.argtypes = [P, c.c_int32, PI32, c.POINTER(c.c_char_p), PC, c.c_int, c.c_int32, c.c_int64, P,
                                    c.c_int32, P, P, P, P]
     L.up_gen_modexp_source.argtypes = [c.c_char_p, c.c_char_p, c.c_int32, c.c_int, c.c_int64, c.c_char_p, c.c_size_t]
@@ -452,6 +455,18 @@ class Context:
                                     _stream_ptr(stream)))
         return out, counts_out, layout
 
+    def eval_tpi(self, op: str, a: Column, b: Column, tpi: int = 1, div_algo: str = "long", out: Optional[Column] = None,
+                 stream=None) -> Column:
+        """a <op> b per row with tpi lanes per row (include/up.h up_eval_tpi);
+        div_algo "long" (Knuth D) or "newton" (Newton-Raphson) for "/"."""
+        p, s = self.expr_type(f"c1{op}c2", [a, b])
+        if out is None:
+            out = Column(p, s, a.n)
+        d, ad, bd = out.desc(), a.desc(), b.desc()
+        _chk(lib().up_eval_tpi(self.h, op.encode(), ctypes.byref(ad), ctypes.byref(bd), tpi,
+                               1 if div_algo == "newton" else 0, ctypes.byref(d), _stream_ptr(stream)))
+        return out
+
     def filter(self, lhs: str, op: str, rhs: str, cols: Sequence[Column], ids=None, stream=None):
         """WHERE lhs <op> rhs (include/up.h up_filter): rows whose predicate is
         false get id -1 in `ids` (int32 device tensor, created as zeros when
@@ -538,6 +553,19 @@ def gen_source(variant: str, expr: str, types: Sequence[tuple], n_global: int = 
             arr[i] = up_column(n_global, ld_for(n_global), p, s, limbs(p), 0, None)
     buf = ctypes.create_string_buffer(1 << 24)
     _chk(lib().up_gen_source(variant.encode(), expr.encode(), arr, len(types), n_global, buf, len(buf)))
+    return buf.value.decode()
+
+
+def gen_tpi_source(op: str, types: Sequence[tuple], tpi: int = 1, div_algo: str = "long",
+                   compact: Optional[Sequence[bool]] = None) -> str:
+    arr = (up_column * 2)()
+    for i, (p, s) in enumerate(types):
+        if compact and compact[i]:
+            arr[i] = up_column(1, compact_bytes(p), p, s, limbs(p), LAYOUT_COMPACT, None)
+        else:
+            arr[i] = up_column(1, 4, p, s, limbs(p), 0, None)
+    buf = ctypes.create_string_buffer(1 << 22)
+    _chk(lib().up_gen_tpi_source(op.encode(), arr, tpi, 1 if div_algo == "newton" else 0, buf, len(buf)))
     return buf.value.decode()
 
 

@@ -112,3 +112,15 @@ def test_group_aggregate_typing_and_kernel_compile(tmp_path):
     log = up.nvrtc_compile(src, str(tmp_path / "g.cubin"))
     regs, spills = _regs(log)
     assert spills == 0, log
+
+
+def test_tpi_kernels_compile_for_sm100a():
+    """Every per-operator TPI kernel shape (NEXT-3) compiles with NVRTC for sm_100a (no GPU)."""
+    from paper_conf_icde_lixylz24_b200 import up
+    for op in "+-*":
+        for tpi in (1, 2, 4, 8, 16, 32):
+            for types, cp in (([(35, 5), (32, 2)], None), ([(153, 7), (154, 0)], [True, False])):
+                up.nvrtc_compile(up.gen_tpi_source(op, types, tpi, compact=cp))
+    for alg in ("long", "newton"):
+        for types in ([(40, 5), (30, 2)], [(200, 50), (200, 50)], [(20, 0), (9, 0)]):
+            up.nvrtc_compile(up.gen_tpi_source("/", types, 1, alg))
