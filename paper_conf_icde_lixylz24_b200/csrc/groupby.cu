@@ -174,8 +174,9 @@ __global__ void __launch_bounds__(1024) k_scan_parts(uint32_t *part, long long n
     uint32_t acc = tot[threadIdx.x];
     for (long long i = lo; i < lo + per && i < np; ++i) { const uint32_t v = part[i]; part[i] = acc; acc += v; }
 }
-__global__ void __launch_bounds__(256) k_scan_apply(const uint32_t *__restrict__ in, uint32_t *__restrict__ out,
-                                                     long long m, const uint32_t *__restrict__ part, int inclusive) {
+// (in and out may be the same array: no __restrict__ -- each element is read before it is written)
+__global__ void __launch_bounds__(256) k_scan_apply(const uint32_t *in, uint32_t *out, long long m,
+                                                     const uint32_t *__restrict__ part, int inclusive) {
     __shared__ uint32_t seg[256];
     const long long c = blockIdx.x, b0 = c * SCAN_CHUNK;
     constexpr int PER = SCAN_CHUNK / 256;   // consecutive elements per thread

@@ -18,8 +18,8 @@
 //  * /: per thread (TPI = 1), Q = trunc(|A| 10^(s2+4) / |B|) (P:L1049-1058,
 //    reading Q4) by Knuth's long division (divmod_mag, the fused kernels' path)
 //    or by Newton-Raphson: the reciprocal of the divisor's top
-//    limbs d^-1_(i+1) = d^-1_i (2 - d d^-1_i) in fixed point from a 64-bit
-//    seed, the quotient estimate (dividend top) x d^-1, then an exact
+//    limbs d^-1_(i+1) = d^-1_i (2 - d d^-1_i) in fixed point (NQ + 2 limbs of
+//    precision) from a 64-bit seed, the quotient estimate (dividend top) x d^-1, then an exact
 //    remainder correction.  Both exact; NR costs more multiplies for the short
 //    typed quotients of DECIMAL division (measured).
 // Values and flags equal up_eval_expr("c1 op c2") on the same columns.
@@ -194,12 +194,13 @@ extern "C" __global__ void __launch_bounds__(256) upk(const up_kparams P) {
 
 // Newton-Raphson division, per thread, exact:
 //   normalise v (top bit of limb NV-1 set) and u by the same shift;
-//   X = floor(B^(2T) / vt) for the divisor's top T = min(NV, NQ + 2) limbs,
-//     seeded from the top 64 bits (X0 = floor((2^128 - 1) / d64) B^(T-2)),
-//     X <- X + X (B^(2T) - vt X) / B^(2T) until converged, then fixed
-//     exactly against the remainder B^(2T) - vt X;
-//   q = (top limbs of u) X / B^(2T), then corrected with the exact remainder
-//     u - q v (a few steps at most).
+//   X = floor(B^K / vt) for the divisor's top T = min(NV, NQ + 2) limbs,
+//     K = T + NQ + 2 (X carries NQ + 2 limbs of the quotient's precision),
+//     seeded from the top 64 bits (X0 = floor((2^128 - 1) / d64) B^(K-T-2)),
+//     X <- X + X (B^K - vt X) / B^K (d^-1 (2 - d d^-1)) until converged, then
+//     fixed exactly against the remainder B^K - vt X;
+//   q = (top limbs of u) X / B^K, then corrected with the exact remainder
+//     u - q v (tools-level model: no correction step was ever needed).
 const char *kNrDiv = R"KERNEL(
 template <int N> __device__ __forceinline__ bool neg_top(const u32 (&a)[N]) { return (a[N - 1] >> 31) != 0u; }
 template <int N> __device__ __forceinline__ void add_to(u32 (&a)[N], const u32 *b, int nb) {
@@ -264,60 +265,62 @@ __device__ __noinline__ u32 nr_divmod(u32 (&q)[XQ], const u32 (&u)[XU], const u3
         return divmod_mag<XN, 1, XQ, false>(q, rr, un, vn);
     } else {
         constexpr int T = XQ + 2 < XV ? XQ + 2 : XV;      // divisor limbs the reciprocal uses
-        constexpr int TX = T + 1;                         // X in (B^T, 2 B^T]
+        constexpr int K = T + XQ + 2;                     // X = floor(B^K / vt) in (B^(XQ+2), 2 B^(XQ+2)]
+        constexpr int TX = XQ + 3;
+        constexpr int NE = K + 2;                         // B^K - vt X, two's complement
         u32 vt[T];
 #pragma unroll
         for (int i = 0; i < T; ++i) vt[i] = vn[XV - T + i];
-        // --- seed: X0 = floor((2^128 - 1) / d64) B^(T-2), d64 = top 64 bits of vt
+        // --- seed: X0 = floor((2^128 - 1) / d64) B^(K-T-2), d64 = top 64 bits of vt
         u32 X[TX];
         zero(X);
         {
             const u64 d64 = ((u64)vt[T - 1] << 32) | vt[T - 2];
             const unsigned __int128 x0 = (~(unsigned __int128)0) / d64;     // in (2^64, 2^65]
-            X[T - 2] = (u32)x0;
-            X[T - 1] = (u32)(x0 >> 32);
-            X[T] = (u32)(x0 >> 64);
+            X[K - T - 2] = (u32)x0;
+            X[K - T - 1] = (u32)(x0 >> 32);
+            X[K - T] = (u32)(x0 >> 64);
         }
-        // --- Newton-Raphson: E = B^(2T) - vt X (signed, 2T+1 limbs), X += X E / B^(2T)
-        constexpr int ITER = (32 * TX <= 128) ? 2 : (32 * TX <= 256) ? 3 : (32 * TX <= 512) ? 4 : (32 * TX <= 1024) ? 5 : 6;
+        // --- Newton-Raphson: E = B^K - vt X, X += X E / B^K (each step doubles the correct bits)
+        constexpr int ITER = (32 * TX <= 128) ? 2 : (32 * TX <= 256) ? 3 : (32 * TX <= 512) ? 4 : (32 * TX <= 1024) ? 5
+                           : (32 * TX <= 2048) ? 6 : 7;
 #pragma unroll 1
         for (int it = 0; it < ITER; ++it) {
-            u32 p[2 * T + 2];
-            mul_mag<T, TX, 2 * T + 2>(p, vt, X);
-            u32 e[2 * T + 2];
+            u32 p[NE];
+            mul_mag<T, TX, NE>(p, vt, X);
+            u32 e[NE];
             zero(e);
-            e[2 * T] = 1u;                                // B^(2T)
-            sub_from(e, p, 2 * T + 2);                    // two's complement, 2T+2 limbs
+            e[K] = 1u;                                    // B^K
+            sub_from(e, p, NE);
             const bool eneg = neg_top(e);
-            if (eneg) { for (int i = 0; i < 2 * T + 2; ++i) e[i] = ~e[i]; inc_n(e); }
-            // X E / B^(2T): only limbs >= 2T of the product matter
-            u32 pe[TX + 2 * T + 2];
-            mul_mag<TX, 2 * T + 2, TX + 2 * T + 2>(pe, X, e);
+            if (eneg) { for (int i = 0; i < NE; ++i) e[i] = ~e[i]; inc_n(e); }
+            u32 pe[TX + NE];
+            mul_mag<TX, NE, TX + NE>(pe, X, e);
             u32 dx[TX + 2];
 #pragma unroll
-            for (int i = 0; i < TX + 2; ++i) dx[i] = pe[2 * T + i];
+            for (int i = 0; i < TX + 2; ++i) dx[i] = pe[K + i];
             u32 Xw[TX + 2];
             zext<TX, TX + 2>(Xw, X);
             if (eneg) sub_from(Xw, dx, TX + 2); else add_to(Xw, dx, TX + 2);
 #pragma unroll
             for (int i = 0; i < TX; ++i) X[i] = Xw[i];
         }
-        // --- exact fix: 0 <= B^(2T) - vt X < vt
+        // --- exact fix: 0 <= B^K - vt X < vt
 #pragma unroll 1
         for (int it = 0; it < 8; ++it) {
-            u32 p[2 * T + 2];
-            mul_mag<T, TX, 2 * T + 2>(p, vt, X);
-            u32 e[2 * T + 2];
+            u32 p[NE];
+            mul_mag<T, TX, NE>(p, vt, X);
+            u32 e[NE];
             zero(e);
-            e[2 * T] = 1u;
-            sub_from(e, p, 2 * T + 2);
+            e[K] = 1u;
+            sub_from(e, p, NE);
             if (neg_top(e)) { dec_n(X); continue; }
-            u32 vte[2 * T + 2];
-            zext<T, 2 * T + 2>(vte, vt);
+            u32 vte[NE];
+            zext<T, NE>(vte, vt);
             if (!lt(e, vte)) { inc_n(X); continue; }
             break;
         }
-        // --- quotient estimate: (un >> 32 (XV - T)) X >> 32 (2T)
+        // --- quotient estimate: (un >> 32 (XV - T)) X >> 32 K
         constexpr int XUT = XQE + T + 1;                  // dividend top limbs (q < B^XQE)
         u32 ut[XUT];
 #pragma unroll
@@ -326,7 +329,7 @@ __device__ __noinline__ u32 nr_divmod(u32 (&q)[XQ], const u32 (&u)[XU], const u3
         mul_mag<XUT, TX, XUT + TX>(pq, ut, X);
         u32 qh[XQE + 1];
 #pragma unroll
-        for (int i = 0; i < XQE + 1; ++i) qh[i] = (2 * T + i < XUT + TX) ? pq[(2 * T + i < XUT + TX) ? 2 * T + i : 0] : 0u;
+        for (int i = 0; i < XQE + 1; ++i) qh[i] = (K + i < XUT + TX) ? pq[(K + i < XUT + TX) ? K + i : 0] : 0u;
         // --- exact correction with the full remainder r = un - qh vn (XN + 1 limbs, signed)
         u32 r[XN + 1];
         zext<XN, XN + 1>(r, un);
