@@ -130,6 +130,7 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
 #pragma unroll
     for (int q = 0; q < RPL; ++q)
         for (int l = b; l < WS; l += G) Ssm[l * RSS + rr0 + q] = 0ull;
+    __syncwarp();   // lane b == 0 of the row group reads (negates) these slots below
     int since_norm = 0;
     u32 acc_neg[RPL];     // SUM: the row slot's accumulator currently holds -(sum)
 #pragma unroll

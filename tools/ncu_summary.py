@@ -95,7 +95,7 @@ def main():
                 return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[u]
             os.makedirs(os.path.dirname(a.traffic_json) or ".", exist_ok=True)
             json.dump({"kernel": f["kernel"], "dram_bytes_per_launch": mb("dram__bytes_read.sum") + mb("dram__bytes_write.sum"),
-                       "source": a.rep, "tag": a.tag}, open(a.traffic_json, "w"), indent=1)
+                       "source": f"profiles/{a.tag}.json (ncu --set full: {os.path.basename(a.rep)})", "tag": a.tag}, open(a.traffic_json, "w"), indent=1)
     os.makedirs(os.path.dirname(f"profiles/{a.tag}.json"), exist_ok=True)
     json.dump(summ, open(f"profiles/{a.tag}.json", "w"), indent=1)
     print(json.dumps(summ, indent=1)[:3000])
