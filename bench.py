@@ -14,7 +14,11 @@ A step = one pass of the whole hot path over the resident columns: the fused
 kernel (+ NCCL all-gather of the partials and the exact combine kernel when
 N > 1).  Inputs are seeded synthetic columns (gen/).  For N > 1 rows are
 sharded (weak scaling: every rank owns `rows` rows; typing uses the global
-row count).  Reported with it: `e2e` (same metric through the C ABI from
+row count).  Steps over resident columns are launched pipelined
+(up_set_pipelined: programmatic dependent launch, each step's kernel may
+start while the previous one finishes; --no-pipelined turns it off) and
+timed with one event pair around the K steps (per step, with the L2 flush
+outside, when the flush is needed).  Reported with it: `e2e` (same metric through the C ABI from
 pinned HOST buffers in the paper's compact row format: H2D + ingestion + SUM
 + D2H of the result in the timed region), `roofline` of the fused kernel, `cpu_baseline` (the CPU oracle as it
 stands on a bounded sample), NVML clocks during the timed region, and
@@ -60,10 +64,11 @@ CONFIGS = {
 }
 
 
-def traffic_key(cfg, rows):
-    """profiles/traffic/<key>.json key: the workload name + rows per GPU."""
+def traffic_key(cfg, rows, layout="planes"):
+    """profiles/traffic/<key>.json key: the workload name + rows per GPU
+    (+ "_compact" for compact-resident columns: a different byte count)."""
     import re
-    return re.sub(r"[^A-Za-z0-9]+", "_", cfg["name"]).strip("_") + f"_{rows}"
+    return re.sub(r"[^A-Za-z0-9]+", "_", cfg["name"]).strip("_") + f"_{rows}" + ("_compact" if layout == "compact" else "")
 
 
 def _peaks():
@@ -482,6 +487,8 @@ def main():
                     help="column storage for the expression configs (1-3): limb planes or the paper's compact rows")
     ap.add_argument("--ref-rows", type=int, default=200_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-pipelined", action="store_true",
+                    help="launch each step's SUM kernel without programmatic dependent launch")
     ap.add_argument("--e2e-steps", type=int, default=0)
     ap.add_argument("--P", type=int, default=0, help="cfg5 digits")
     ap.add_argument("--bits", type=int, default=0, help="cfg4 modulus bits")
@@ -551,6 +558,14 @@ def main():
         flush_rd = torch.zeros(int(256e6) // 4, dtype=torch.float32, device="cuda")
         flush_sum = torch.empty((), dtype=torch.float32, device="cuda")
 
+    # Pipelined SUM launches (up_set_pipelined): consecutive steps
+    # are queries over the same resident columns, so each step's kernel may
+    # start streaming while the previous step's kernel finishes.  Not with the
+    # L2 flush (the flush must complete before the step) nor for e2e (the
+    # ingestion kernel right before the SUM writes its inputs).
+    pipelined = flush is None and not args.no_pipelined
+    ctx.set_pipelined(pipelined)
+
     def step():
         ss()
 
@@ -576,47 +591,80 @@ def main():
             torch.cuda.synchronize()
     torch.cuda.synchronize()
 
-    # ---- timed region: K steps, barrier + sync on both sides, CUDA events
+    # ---- timed region: K steps between a barrier + sync on both sides; CUDA
+    # events on the launching stream.  Without an L2 flush: ONE event pair
+    # around the K steps (events between steps would serialise them); with the
+    # flush (cfg1 at 1M rows): an event pair around each step, the flush outside.
     K = args.steps
-    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
-    sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+
+    def body():
+        wl.kernel(partial)
+        if ws > 1:     # the exchange step of ShardedSum.__call__
+            dist.all_gather_into_tensor(ss.gathered, partial)
+            ctx.sum_combine(ss.gathered, LA, out=ss.total)
+
+    def ev():
+        return torch.cuda.Event(enable_timing=True)
+
     l0 = ctx.launches
     if ws > 1:
         dist.barrier()
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
-        for i in range(K):
-            if flush is not None:
+        if flush is None:
+            e0, e1 = ev(), ev()
+            e0.record(stream)
+            for i in range(K):
+                body()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1)
+        else:
+            sev = [(ev(), ev()) for _ in range(K)]
+            for i in range(K):
                 flush.zero_()            # evict the inputs from L2 (outside the step's events)
                 torch.sum(flush_rd, dim=0, out=flush_sum)
-            sev[i][0].record(stream)
-            kev[i][0].record(stream)
-            wl.kernel(partial)
-            kev[i][1].record(stream)
-            if ws > 1:     # the exchange step of ShardedSum.__call__ (split out to time the kernel alone)
-                dist.all_gather_into_tensor(ss.gathered, partial)
-                ctx.sum_combine(ss.gathered, LA, out=ss.total)
-            sev[i][1].record(stream)
-        torch.cuda.synchronize()
+                sev[i][0].record(stream)
+                body()
+                sev[i][1].record(stream)
+            torch.cuda.synchronize()
+            ms = sum(a.elapsed_time(b) for a, b in sev)
     if ws > 1:
         dist.barrier()
     launches = ctx.launches - l0
-    ms = sum(a.elapsed_time(b) for a, b in sev)
-    kernel_ms = sum(a.elapsed_time(b) for a, b in kev) / K
     if ws > 1:
         t = torch.tensor([ms], dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     ms_per_step = ms / K
     value = n_global / (ms_per_step / 1e3)
+    # the dominant kernel's average launch duration: when a step IS one launch
+    # (N = 1, one fused kernel), the timed region's events give it directly
+    # (ms / K); otherwise a second K-step pass with events around the kernel
+    if ws == 1 and launches == K:
+        kernel_ms, kernel_src = ms_per_step, "timed region: step = one launch (events around the K steps) / K"
+    else:
+        kev = [(ev(), ev()) for _ in range(K)]
+        torch.cuda.synchronize()
+        for i in range(K):
+            if flush is not None:
+                flush.zero_()
+                torch.sum(flush_rd, dim=0, out=flush_sum)
+            kev[i][0].record(stream)
+            wl.kernel(partial)
+            kev[i][1].record(stream)
+        torch.cuda.synchronize()
+        kernel_ms = sum(a.elapsed_time(b) for a, b in kev) / K
+        kernel_src = "second K-step pass, events around the kernel launch"
     ctx.check()
     result = ss.result()
     peaks = _peaks()
     roofline = wl.roofline(kernel_ms, peaks)
+    roofline["kernel_ms_source"] = kernel_src
     # traffic = dram__bytes_read + dram__bytes_write of the dominant kernel per
     # launch, from one `ncu --set full` capture of THIS workload (same config,
     # precision and rows per GPU), summarised by tools/ncu_summary.py
-    tkey = traffic_key(cfg, rows)
+    tkey = traffic_key(cfg, rows, args.layout)
     tp = os.path.join(ROOT, "profiles", "traffic", f"{tkey}.json")
     roofline["traffic"] = None
     roofline["traffic_key"] = tkey
@@ -628,7 +676,9 @@ def main():
         except Exception:
             pass
 
-    # ---- e2e through the C ABI from pinned host buffers
+    # ---- e2e through the C ABI from pinned host buffers (ingestion writes the
+    # columns the SUM reads next: not pipelined)
+    ctx.set_pipelined(False)
     host = wl.e2e_host_buffers()
     torch.cuda.synchronize()
     res_host = torch.empty(LA, dtype=torch.int32, pin_memory=True)
@@ -683,6 +733,7 @@ def main():
         desc.update(wl.workload_desc())
         if cfg["kind"] == "expr":
             desc["layout"] = args.layout
+        desc["pipelined"] = pipelined
         line = {
             "metric": METRIC, "value": value, "unit": "tuples/s", "n_gpus": ws, "steps": K,
             "warmup": args.warmup, "warmup_extra_untimed": warm_extra, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": scaling,

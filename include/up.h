@@ -54,6 +54,20 @@ up_status up_ctx_create(int device, up_ctx **out);
 up_status up_ctx_destroy(up_ctx *ctx);
 
 /*
+ * Pipelined SUM launches (default off).  When on, the fused SUM kernels of
+ * up_sum_expr / up_sum are launched with programmatic dependent launch: their
+ * CTAs may start (and stream their input columns) while the previous kernel
+ * on the same stream is finishing, and wait for that kernel to complete
+ * before touching the context's SUM workspace and d_partial.  Back-to-back
+ * aggregation queries over resident columns then overlap one query's ramp
+ * with the previous one's tail.  Contract: the kernel immediately before such
+ * a SUM on its stream must not write that SUM's input columns (a kernel two
+ * or more launches back is fully ordered as usual).  Turn it off around
+ * ingestion or evaluation that produces a column a SUM reads next.
+ */
+up_status up_set_pipelined(up_ctx *ctx, int on);
+
+/*
  * A DECIMAL(p,s) column of n rows as `limbs` limb planes (SURVEY §8a layout):
  * data[j*ld + i] is limb j (little-endian, 32-bit) of row i's mantissa in
  * TWO'S COMPLEMENT, value = mantissa * 10^-s (Eq. 1).  ld >= n is a

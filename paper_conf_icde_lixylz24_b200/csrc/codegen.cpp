@@ -285,6 +285,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     k << "extern \"C\" __global__ void " << launch_bounds(256, min_blocks) << " upk(const up_kparams P) {\n";
     k << "    constexpr int R = " << R << ";\n";
     k << "    u32 fl = 0;\n";
+    if (opt.sum) k << "    griddep_launch_dependents();\n";
     if (opt.sum) {
         if (cs) k << "    AccCS<" << LOUT << "> acc; acc.init();\n";
         else k << "    AccChain<" << LOUT << "," << KC << "> acc; acc.init();\n";
@@ -422,6 +423,10 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     k << "    }\n";
     k << "    if (fl) atomicOr(P.flags, fl);\n";
     if (opt.sum) {
+        // the SUM workspace / ticket / result of the previous launch on this
+        // stream are re-used: wait for it (no-op without a PDL launch)
+        k << "    griddep_wait();\n";
+        info.pdl = true;
         k << "    __shared__ u64 sm[(256 / 32) * " << (NS + 1) << "];\n";
         k << "    u64 vals[" << (NS + 1) << "];\n";
         if (cs) {

@@ -26,6 +26,7 @@ struct GenInfo {
     int dyn_smem = 0;        // dynamic shared memory per block (bytes)
     int threads = 256;
     int rows_per_block = 0;  // > 0: rows handled per block-iteration (warp-per-row kernels)
+    bool pdl = false;        // kernel waits (griddepcontrol.wait) before touching its SUM workspace
 };
 
 std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, const GenOpts &opt, GenInfo &info);

@@ -67,6 +67,7 @@ struct Drv {
     CUresult (*OccupancyMaxActiveBlocksPerMultiprocessor)(int *, CUfunction, int, size_t) = nullptr;
     CUresult (*GetErrorString)(CUresult, const char **) = nullptr;
     CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
+    CUresult (*LaunchKernelEx)(const CUlaunchConfig *, CUfunction, void **, void **) = nullptr;
     bool ok = false;
 } drv;
 
@@ -86,6 +87,7 @@ cudaError_t load_drv() {
     UP_ENTRY("cuOccupancyMaxActiveBlocksPerMultiprocessor", OccupancyMaxActiveBlocksPerMultiprocessor);
     UP_ENTRY("cuGetErrorString", GetErrorString);
     UP_ENTRY("cuFuncSetAttribute", FuncSetAttribute);
+    UP_ENTRY("cuLaunchKernelEx", LaunchKernelEx);
 #undef UP_ENTRY
     drv.ok = true;
     return cudaSuccess;
@@ -131,6 +133,7 @@ struct JitKernel {
     int threads = kThreads;
     int dyn_smem = 0;      // dynamic shared memory per block (bytes)
     int rows_per_block = 0;  // > 0: warp-per-row kernels (rows per block-iteration)
+    bool pdl = false;        // may be launched with programmatic stream serialization
     std::string src;
 };
 
@@ -165,6 +168,7 @@ struct up_ctx {
     std::unordered_map<std::string, SplitPlan> plans;   // split SUM plans (up_sum_expr)
     uint64_t launches = 0;
     double jit_ms = 0.0;
+    bool pipelined = false;   // up_set_pipelined: PDL launches of the fused SUM kernels
     std::mutex mu;
 };
 
@@ -363,7 +367,21 @@ up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream
     long long cap = (long long)k->blocks_per_sm * c->num_sms;
     int grid = (int)std::max(1ll, std::min(want, cap));
     void *args[] = {&P};
-    CU_TRY(drv.LaunchKernel(k->fn, grid, 1, 1, k->threads, 1, 1, (unsigned)k->dyn_smem, (CUstream)st, args, nullptr));
+    if (k->pdl && c->pipelined) {
+        CUlaunchAttribute at[1];
+        at[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+        at[0].value.programmaticStreamSerializationAllowed = 1;
+        CUlaunchConfig cfg = {};
+        cfg.gridDimX = grid; cfg.gridDimY = 1; cfg.gridDimZ = 1;
+        cfg.blockDimX = k->threads; cfg.blockDimY = 1; cfg.blockDimZ = 1;
+        cfg.sharedMemBytes = (unsigned)k->dyn_smem;
+        cfg.hStream = (CUstream)st;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        CU_TRY(drv.LaunchKernelEx(&cfg, k->fn, args, nullptr));
+    } else {
+        CU_TRY(drv.LaunchKernel(k->fn, grid, 1, 1, k->threads, 1, 1, (unsigned)k->dyn_smem, (CUstream)st, args, nullptr));
+    }
     c->launches++;
     return UP_OK;
 }
@@ -404,6 +422,7 @@ up_status expr_kernel(up_ctx *c, const char *expr, const up_column *cols, int nc
     k->rows_per_thread = info.rows_per_thread;
     k->ws_slots = info.ws_slots;
     k->rows_per_block = info.rows_per_block;
+    k->pdl = info.pdl;
     if (info.threads != k->threads || info.dyn_smem != k->dyn_smem) {
         k->threads = info.threads;
         if (info.dyn_smem > 0)
@@ -484,6 +503,12 @@ up_status up_ctx_create(int device, up_ctx **out) {
     CUDA_TRY(cudaMemset(c->d_flags, 0, 64));
     CUDA_TRY(cudaDeviceSynchronize());
     *out = c.release();
+    return UP_OK;
+}
+
+up_status up_set_pipelined(up_ctx *c, int on) {
+    if (!c) return fail(UP_E_INVAL, "null ctx");
+    c->pipelined = on != 0;
     return UP_OK;
 }
 

@@ -41,7 +41,7 @@ EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_l
            "up_column_from_host_compact", "up_column_from_device_compact", "up_column_to_host_compact",
            "up_expr_optimized", "up_gen_contract_source", "up_agg_type", "up_group_aggregate",
            "up_gen_group_agg_source", "up_filter", "up_group_ids", "up_group_combine", "up_eval_tpi",
-           "up_gen_tpi_source"]
+           "up_gen_tpi_source", "up_set_pipelined"]
 
 AGG = {"SUM": 0, "MIN": 1, "MAX": 2, "AVG": 3}
 
@@ -63,6 +63,7 @@ def lib():
     L.up_sum_precision.argtypes = [c.c_int32, c.c_int64]; L.up_sum_precision.restype = c.c_int32
     L.up_ctx_create.argtypes = [c.c_int, c.POINTER(P)]
     L.up_ctx_destroy.argtypes = [P]
+    L.up_set_pipelined.argtypes = [P, c.c_int]
     L.up_column_from_host_bin.argtypes = [P, P, c.c_int32, P, PC, P]
     L.up_column_from_device_bin.argtypes = [P, P, c.c_int32, P, PC, P]
     L.up_column_from_host.argtypes = [P, c.POINTER(c.c_char_p), PC, P]
@@ -221,6 +222,13 @@ class Context:
         except Exception:
             pass
 
+    def set_pipelined(self, on: bool = True):
+        """Programmatic dependent launch of the fused SUM kernels (up.h
+        up_set_pipelined): back-to-back SUMs over resident columns overlap.
+        The kernel right before such a SUM on its stream must not write the
+        SUM's input columns."""
+        _chk(lib().up_set_pipelined(self.h, 1 if on else 0))
+
     # ------------------------------------------------------------------ info
     @property
     def launches(self) -> int:
@@ -347,9 +355,9 @@ class Context:
 
     def sum_expr(self, expr: str, cols: Sequence[Column], n_global: int = 0, out=None, stream=None):
         """SELECT SUM(expr): returns the device tensor of LA two's-complement limbs."""
-        import torch
-        _, _, LA = self.sum_type(expr, cols, n_global)
-        if out is None:
+        if out is None:     # (typing parses the expression: only when the caller has no buffer)
+            import torch
+            _, _, LA = self.sum_type(expr, cols, n_global)
             out = torch.empty(LA, dtype=torch.int32, device=cols[0].data.device)
         _chk(lib().up_sum_expr(self.h, expr.encode(), _descs(cols), len(cols), n_global, out.data_ptr(),
                                _stream_ptr(stream)))
