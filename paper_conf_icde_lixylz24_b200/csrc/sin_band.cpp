@@ -232,7 +232,9 @@ extern "C" __global__ void __launch_bounds__(32) upk(const up_kparams P) {
                 r1[q] = r0[q] = qprev[q] = p0a[q] = p0b[q] = p1a[q] = Alo[q] = 0u;
                 ynext[q] = lds32p(ld0, yl + 4u * q);
             }
-#pragma unroll 1
+            // unrolled by 2: the digit-history rotation (p0b <- p0a <- p0, Alo) becomes
+            // register renaming instead of moves (SASS: 84 -> 76 instructions per step)
+#pragma unroll 2
             for (int tau = 0; tau < steps; ++tau) {
                 const int j = jb - tau;
                 const bool act = (unsigned)j <= (unsigned)jtop;
