@@ -74,6 +74,6 @@ struct SinBandInfo {
     int G = 0, rows_per_block = 0, smem = 0, ws_slots = 0, delta = 0, W = 0;
 };
 std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum, int G_req, SinBandInfo &info,
-                                std::string &err, int rpl_req = 0);
+                                std::string &err);
 
 }  // namespace uph

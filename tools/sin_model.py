@@ -6,7 +6,8 @@ CUDA code.  It is NOT the oracle: it mirrors the kernel's 32-bit digit steps
 3-by-2 quotient steps against a normalised 64-bit divisor, the bit offset o_k
 that absorbs the 2^(2s) factor of 10^(2s), digit drops, the low-bit mask, the
 scaled carry-save running sum) so a mistake in that plan shows up as a
-mismatch against the Q13 definition (tests/test_sin_model.py).
+mismatch against the Q13 definition (tests/test_sin_model.py); term_divide64
+is the same division on 64-bit chunks (the band kernel's digit pairs).
 
 Per row, x = m 10^-s (|m| < 10^9, 2s < 32), X2 = m^2,
 D_k = 5^(2s) (2k)(2k+1), 10^(2s) (2k)(2k+1) = 2^(2s) D_k.
@@ -107,7 +108,86 @@ def term_divide(Y, X2, D, n_out):
     return q[:n_out], rare
 
 
-def sin_row(m: int, s: int, P: int, c_scale=None, check=True):
+M64 = (1 << 64) - 1
+C64 = 1 << 64
+
+
+def mg_reciprocal_2by1_64(d: int) -> int:
+    """v = floor((C^2 - 1) / d) - C for a normalised 64-bit d (MG 2011, 2-by-1)."""
+    assert d >> 63 == 1
+    return (C64 * C64 - 1) // d - C64
+
+
+def mg_div_2by1_64(u1, u0, d, v):
+    """Moller-Granlund 2011, Algorithm 4 on 64-bit words: (q, r), u1 < d."""
+    assert u1 < d
+    q = v * u1 + ((u1 << 64) | u0)
+    q1, q0 = (q >> 64) & M64, q & M64
+    q1 = (q1 + 1) & M64
+    r = (u0 - q1 * d) & M64
+    if r > q0:
+        q1 = (q1 - 1) & M64
+        r = (r + d) & M64
+    if r >= d:
+        q1 += 1
+        r -= d
+    return q1, r
+
+
+def term_divide64(Y, X2, D, n_out):
+    """The 64-bit-chunk variant (sin_band.cpp, band64): chunks c_m = y_2m +
+    y_(2m+1) B, c_m X2 = L_m + H_m C (C = 2^64), A_m = L_m + H_(m-1) (65
+    bits, no carry travels), V_m = lo64(A_m << sh) + (A_(m-1) >> (64 - sh))
+    (sh = clz64(D), 0..63; carry <= 1 into the position above: Horner, added
+    to R), one 2-by-1 step on 64-bit words per chunk.  Returns 32-bit
+    quotient digits."""
+    sh = 64 - D.bit_length()
+    Dn = D << sh
+    v = mg_reciprocal_2by1_64(Dn)
+    n = len(Y)
+    nc = (n + 1) // 2
+    def chunk(m):
+        if m < 0 or m >= nc:
+            return 0
+        lo = Y[2 * m] if 2 * m < n else 0
+        hi = Y[2 * m + 1] if 2 * m + 1 < n else 0
+        return lo | (hi << 32)
+    def LH(m):
+        pr = chunk(m) * X2
+        return pr & M64, pr >> 64
+    def A(m):
+        return LH(m)[0] + LH(m - 1)[1]          # < 2^64 + 2^60
+    def Vc(m):
+        t = ((A(m) << sh) & M64) + (A(m - 1) >> (64 - sh))
+        assert t >> 64 <= 1
+        return t & M64, t >> 64
+    top = nc + 2
+    R = 0
+    q = [0] * (top + 2)
+    rare = False
+    for m in range(top, -1, -1):
+        u0, c = Vc(m)
+        T = R + c
+        assert T < C64
+        if T >= Dn:
+            rare = True
+            T -= Dn
+            j = m + 1
+            while True:
+                q[j] += 1
+                if q[j] < C64:
+                    break
+                q[j] = 0
+                j += 1
+        q[m], R = mg_div_2by1_64(T, u0, Dn, v)
+    out = []
+    for x in q:
+        out += [x & M32, x >> 32]
+    out += [0] * max(0, n_out - len(out))
+    return out[:n_out], rare
+
+
+def sin_row(m: int, s: int, P: int, c_scale=None, check=True, chunk64=False):
     """sin_P(m 10^-s) per the kernel's plan; returns the integer mantissa at scale P."""
     X2 = m * m
     W = (abs(m) * 10 ** (P - s)).bit_length() // 32 + 3
@@ -124,7 +204,7 @@ def sin_row(m: int, s: int, P: int, c_scale=None, check=True):
         Sacc += sign * (Yv << (c - o))
         D = 5 ** (2 * s) * (2 * k) * (2 * k + 1)
         assert D < 1 << 64
-        q, rare = term_divide(Y, X2, D, len(Y) + 2)
+        q, rare = (term_divide64 if chunk64 else term_divide)(Y, X2, D, len(Y) + 2)
         rare_any |= rare
         if check:
             assert from_digits(q) == (Yv * X2) // D
@@ -160,6 +240,7 @@ if __name__ == "__main__":
         for s in (0, 2, 8):
             for _ in range(20):
                 m = rng.randrange(-(10 ** (s + 1)) + 1, 10 ** (s + 1))
-                got, _ = sin_row(m, s, P)
-                assert got == sin_q13(m, s, P), (m, s, P)
+                for c64 in (False, True):
+                    got, _ = sin_row(m, s, P, chunk64=c64)
+                    assert got == sin_q13(m, s, P), (m, s, P, c64)
     print("model == Q13")
