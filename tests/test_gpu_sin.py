@@ -89,9 +89,11 @@ def test_sin_odd_symmetry_on_gpu():
 @pytest.mark.parametrize("pst", [(9, 8), (8, 7), (3, 2), (1, 0)])
 def test_sin_register_sum_variant(P, n, pst):
     """The default kernel for W <= 200 limbs (t in shared memory, S in
-    registers, one 3-by-2 division pass per term) against the oracle:
-    scales whose constant shift is a right shift (s = 8, 7), a left shift
-    (s = 2) or absent with no constant divisor (s = 0)."""
+    registers, one division pass per term: 64-bit 2-by-1 steps on limb
+    pairs, one 3-by-2 step first for an odd limb count; 32-bit 2-by-1 steps
+    while D_k < 2^32) against the oracle: scales whose constant shift is a
+    right shift (s = 8, 7), a left shift (s = 2) or absent with no constant
+    divisor (s = 0); row counts and P give odd and even limb counts."""
     p, s = pst
     mag, neg = synth.uniform_decimal(n, p, 5, 4)
     c = G.ctx()
