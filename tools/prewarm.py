@@ -43,6 +43,20 @@ def sources():
         N, _, _ = synth.rsa_modulus(bits)
         for e in (3, 65537):
             out.append(up.gen_modexp_source(e, N, len(str(N)), False, n))
+    # the slowest compiles of the suite: 2048-bit Montgomery kernels (radix 2^28 default,
+    # and the 32-bit CIOS that test_modexp_parity forces with UP_MONT32)
+    N, _, _ = synth.rsa_modulus(2048)
+    for e in (3, 65537):
+        out.append(up.gen_modexp_source(e, N, len(str(N)), False, 333))
+    os.environ["UP_MONT32"] = "1"
+    for bits in (1024, 1034, 2048):
+        N, _, _ = synth.rsa_modulus(bits)
+        for e in (3, 65537):
+            out.append(up.gen_modexp_source(e, N, len(str(N)), False, 333))
+    del os.environ["UP_MONT32"]
+    N, _, _ = synth.rsa_modulus(1034)
+    for e in (3, 65537):
+        out.append(up.gen_modexp_source(e, N, len(str(N)), False, 333))
     N, _, _ = synth.rsa_modulus(1024)
     out.append(up.gen_modexp_source(65537, N, len(str(N)), True, 10_000_000))
     out.append(up.gen_modexp_source(65537, N, len(str(N)), False, 10_000_000))
