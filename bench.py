@@ -656,6 +656,26 @@ def main():
         torch.cuda.synchronize()
         kernel_ms = sum(a.elapsed_time(b) for a, b in kev) / K
         kernel_src = "second K-step pass, events around the kernel launch"
+    # the same K steps without programmatic dependent launch (reported beside the
+    # pipelined value: what each step costs when launches are fully serialised)
+    ms_unpiped = None
+    if pipelined:
+        ctx.set_pipelined(False)
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        u0, u1 = ev(), ev()
+        u0.record(stream)
+        for i in range(K):
+            body()
+        u1.record(stream)
+        torch.cuda.synchronize()
+        ms_unpiped = u0.elapsed_time(u1) / K
+        if ws > 1:
+            t = torch.tensor([ms_unpiped], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms_unpiped = float(t.item())
+        ctx.set_pipelined(True)
     ctx.check()
     result = ss.result()
     peaks = _peaks()
@@ -734,6 +754,8 @@ def main():
         if cfg["kind"] == "expr":
             desc["layout"] = args.layout
         desc["pipelined"] = pipelined
+        if ms_unpiped is not None:
+            desc["not_pipelined"] = {"ms_per_step": ms_unpiped, "value": n_global / (ms_unpiped / 1e3)}
         line = {
             "metric": METRIC, "value": value, "unit": "tuples/s", "n_gpus": ws, "steps": K,
             "warmup": args.warmup, "warmup_extra_untimed": warm_extra, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": scaling,

@@ -44,15 +44,16 @@ namespace uph {
 
 namespace {
 
-// bank-conflict-minimising padded row stride (words) for lanes (r, b) that
-// touch word (base - DELTA b) of row r; elt = 1 (u32) or 2 (u64 words)
-int pick_stride(int R, int G, int DELTA, int elt, int RPL) {   // DELTA here: digit distance between lanes
+// bank-conflict-minimising padded row stride (words) for one access
+// instruction of the warp: lane (g, b) touches word (base - D b) of row slot g
+// (D = digit distance between consecutive band lanes); elt = 1 (u32) or 2 (u64)
+int pick_stride(int R, int G, int D, int elt) {
     int best = R, bestc = 1 << 30;
     for (int rs = R; rs < R + 64; ++rs) {
         int cnt[32] = {0};
-        for (int b = 0; b < G; ++b)              // one access instruction: row slots g RPL + q, q fixed
+        for (int b = 0; b < G; ++b)
             for (int g = 0; g < 32 / G; ++g) {
-                const long long idx = (long long)(1000 - DELTA * b) * rs + g * RPL;
+                const long long idx = (long long)(1000 - D * b) * rs + g;
                 for (int e = 0; e < elt; ++e) cnt[(idx * elt + e) & 31]++;
             }
         int mx = 0;
@@ -79,7 +80,7 @@ std::string hex_arr(const std::vector<uint32_t> &w) {
 // against D~ = D_k 2^sh.  Half the steps of the 32-bit band for the same
 // digits; the offsets o_k, drops and masks stay per 32-bit digit (quotient
 // digit i goes to Y digit i - drop).  tools/sin_model.py::term_divide64 is
-// the word-level model.  One row per lane group (RPL = 1).
+// the word-level model.  One row per lane group.
 const char *kBand64Body = R"KERNEL(
 extern __shared__ __align__(16) u64 Ssm[];
 #define YSM (reinterpret_cast<u32 *>(Ssm + WS * RSS))
@@ -397,7 +398,7 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
     if (!split) NR = (int)std::max(1.0, std::floor(std::pow(2.0, 61.0 - per_row)));
     else NR = (int)std::max(1.0, std::floor(std::pow(2.0, 61.0 - (std::log2((double)kmax + G) + 33))));
     // lanes of one step touch digits 2 DELTA apart (lane b) in rows g
-    const int RSY = pick_stride(R, G, 2 * DELTA, 1, 1), RSS = pick_stride(R, G, 2 * DELTA, 2, 1);
+    const int RSY = pick_stride(R, G, 2 * DELTA, 1), RSS = pick_stride(R, G, 2 * DELTA, 2);
     // negative (even-k) terms have o_k = c for every even k (s = 8: o = 16; s = 0: o = 0)
     bool negsh0 = true;
     for (int kk = 2; kk <= 64; kk += 2) negsh0 = negsh0 && (((2 * s * (kk - 1)) & 31) == csc);
