@@ -68,7 +68,7 @@ def traffic_key(cfg, rows, layout="planes"):
     """profiles/traffic/<key>.json key: the workload name + rows per GPU
     (+ "_compact" for compact-resident columns: a different byte count)."""
     import re
-    return re.sub(r"[^A-Za-z0-9]+", "_", cfg["name"]).strip("_") + f"_{rows}" + ("_compact" if layout == "compact" else "")
+    return re.sub(r"[^A-Za-z0-9]+", "_", cfg["name"]).strip("_") + f"_{rows}" + ("" if layout == "planes" else "_" + layout)
 
 
 def _peaks():
@@ -147,6 +147,11 @@ class Workload:
         self.e2e_rows = min(rows, E2E_MAX_ROWS)
 
 
+def _col_bytes(p, layout):
+    from paper_conf_icde_lixylz24_b200 import up
+    return {"compact": up.compact_bytes(p), "quads": 16 * up.quads(p)}.get(layout, 4 * up.limbs(p))
+
+
 class ExprWorkload(Workload):
     def setup(self):
         from gen import device as gdev
@@ -162,9 +167,9 @@ class ExprWorkload(Workload):
         self.P, self.S, self.LA = ctx.sum_type(cfg["expr"], self.cols, self.n_global)
         self.e2e_cols = [up.Column(p, s, self.e2e_rows, layout=self.args.layout) for p, s in cfg["types"]]
         # algorithmic bytes per row: the columns as stored -- limb planes (4 B per
-        # limb) or the paper's compact rows (Lb bytes)
-        self.bytes_per_row = sum((up.compact_bytes(p) if self.args.layout == "compact" else 4 * up.limbs(p))
-                                 for p, s in cfg["types"])
+        # limb), the paper's compact rows (Lb bytes) or limb quads
+        # (16 B per quad, the sign-flag limb and padding included)
+        self.bytes_per_row = sum(_col_bytes(p, self.args.layout) for p, s in cfg["types"])
 
     def kernel(self, out):
         self.ctx.sum_expr(self.cfg["expr"], self.cols, self.n_global, out=out)
@@ -207,7 +212,7 @@ class ExprWorkload(Workload):
         ach = alg / (kernel_ms / 1e3) / 1e9
         r = {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
              "frac": round(ach / peak, 4), "kernel_ms": round(kernel_ms, 5), "alg_bytes_per_launch": alg,
-             "alg_unit": f"{self.bytes_per_row} B/row ({'compact rows' if self.args.layout == 'compact' else 'limb planes'}"
+             "alg_unit": f"{self.bytes_per_row} B/row ({self.args.layout} layout"
                          f" of all columns) x {self.rows} rows",
              "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks
              else "fallback 6.65 TB/s"}
@@ -244,7 +249,8 @@ class ExprWorkload(Workload):
         t_tc = self._time(lambda: self.ctx.sum_expr("c1*c2", [c1, c2], self.n_global, out=out))
         t_rest = self._time(lambda: self.ctx.sum_expr("c1/c2", [c3, c4], self.n_global, out=out))
         peak = peaks.get("hbm_gbs", 6650.0)
-        tc_bytes = 2 * 4 * L * self.rows
+        tc_row = _col_bytes(p, self.args.layout)
+        tc_bytes = 2 * tc_row * self.rows
         ach = tc_bytes / (t_tc / 1e3) / 1e9
         mag = lambda k: max(1, (10 ** k).bit_length() // 32 + 1)   # noqa: E731
         nu = mag(p + s + 4)
@@ -253,10 +259,11 @@ class ExprWorkload(Workload):
         rest_ach = div_products * self.rows / (t_rest / 1e3)
         return {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
                 "kernel_ms": round(t_tc, 5), "alg_bytes_per_launch": tc_bytes,
-                "alg_unit": f"contraction kernel: c1, c2 limb planes {2 * 4 * L} B/row x {self.rows} rows",
+                "alg_unit": f"contraction kernel: c1, c2 as stored ({self.args.layout}) {2 * tc_row} B/row x {self.rows} rows",
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s",
                 "kernels": [
-                    {"kernel": "k_contract_tc (SUM(c1*c2), tcgen05 kind::i8)", "ms": round(t_tc, 5), "bound": "hbm",
+                    {"kernel": ("k_contract_tq" if self.args.layout == "quads" else "k_contract_tc") +
+                               " (SUM(c1*c2), tcgen05 kind::i8)", "ms": round(t_tc, 5), "bound": "hbm",
                      "alg_bytes": tc_bytes, "achieved_gbs": round(ach, 1), "frac": round(ach / peak, 4)},
                     {"kernel": "upk rest (SUM(-c3/c4), top-limb division)", "ms": round(t_rest, 5), "bound": "alu",
                      "alg_products": div_products * self.rows,
@@ -483,7 +490,7 @@ def main():
     ap.add_argument("--rows", type=int, default=0, help="rows per GPU (default: the config's)")
     ap.add_argument("--global-rows", type=int, default=0, help="total rows, sharded over the GPUs (strong scaling)")
     ap.add_argument("--impl", default="up", choices=["up", "reference"])
-    ap.add_argument("--layout", default="planes", choices=["planes", "compact"],
+    ap.add_argument("--layout", default="planes", choices=["planes", "compact", "quads"],
                     help="column storage for the expression configs (1-3): limb planes or the paper's compact rows")
     ap.add_argument("--ref-rows", type=int, default=200_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -94,11 +94,28 @@ typedef struct {
  *     (+ range check), the _bin / string calls convert.  Other entry points
  *     return UP_E_UNSUPPORTED for compact inputs.
  */
-enum { UP_LAYOUT_PLANES = 0, UP_LAYOUT_COMPACT = 1 };
+/*
+ *  UP_LAYOUT_QUADS -- limb quads: the limbs grouped four at a time per row,
+ *     G = up_quads(p) = ceil((limbs + 1) / 4) quads of ld rows; quad g of row i
+ *     is the 16 bytes ((uint32_t *)data)[4*(g*ld + i) .. +4) = limbs 4g..4g+3
+ *     (two's complement as in the planes), limb `limbs` holds the SIGN FLAG
+ *     (1 for a negative row, else 0) and the limbs above it are 0.  ld >= n,
+ *     a multiple of 4; data 16-byte aligned, G*ld*16 bytes.  Why: a 3-D TMA
+ *     box of this layout lands in shared memory as the tensor cores' MN-major
+ *     core matrices (16 digit bytes x 8 rows) with the sign digit included,
+ *     so SUM(c_a*c_b) feeds tcgen05 straight from the copies (SURVEY §8a rows
+ *     a6/a11; contract_tc.cu).  Read by up_eval_expr / up_sum_expr / up_sum /
+ *     up_filter (every generated kernel reads quads with 16-byte loads);
+ *     ingestion and read-back convert through limb planes in the ctx scratch.
+ *     Other entry points return UP_E_UNSUPPORTED for quad inputs.
+ */
+enum { UP_LAYOUT_PLANES = 0, UP_LAYOUT_COMPACT = 1, UP_LAYOUT_QUADS = 2 };
 
 /* Limb count L = min{L : 10^p <= 2^(32L-1)} (reading Q1 of P:L821-837 vs
  * reproduces 18/38/76/153/307 <-> 2/4/8/16/32). */
 int32_t up_limbs(int32_t p);
+/* Quads of a UP_LAYOUT_QUADS column: ceil((up_limbs(p) + 1) / 4). */
+int32_t up_quads(int32_t p);
 /* ld for n rows (n rounded up to a multiple of 4). */
 int64_t up_ld(int64_t n);
 /* SUM result precision p + ceil(log10 N), N = n_global (reading Q9). */

@@ -11,6 +11,7 @@
 
 #include <cstdlib>
 #include <functional>
+#include <map>
 #include <sstream>
 
 namespace uph {
@@ -73,20 +74,46 @@ struct Emitter {
     std::ostringstream o;
     int tmp = 0;
     std::vector<bool> lazy;   // column c is read from global memory by the divisions that use it
+    std::vector<bool> quad;   // column c is stored as limb quads (limb j at g + (j>>2)*l + (j&3))
     std::string fresh(const char *pfx) { return std::string(pfx) + std::to_string(tmp++); }
     bool is_lazy(const Node *n) const { return n->op == Op::Col && (size_t)n->col < lazy.size() && lazy[(size_t)n->col]; }
     // limb j (static) of operand n: register array x, or a global load for a lazy column
     std::string limb(const Node *n, const std::string &x, int j) const {
-        if (is_lazy(n)) return "__ldg(g" + std::to_string(n->col) + " + (long long)" + std::to_string(j) + " * l" + std::to_string(n->col) + ")";
+        if (is_lazy(n)) return "__ldg(g" + std::to_string(n->col) + " + " + lazy_off(n->col, j) + ")";
         return x + "[" + std::to_string(j) + "]";
+    }
+    // limb j of the decision window: for a lazy limb-quad column the window's
+    // quads are loaded once with 16-byte loads (and shared by the two operands
+    // when they are the same column)
+    std::map<std::pair<int, int>, std::string> wq;   // (column, quad) -> uint4 of this division's window
+    std::string top_limb(const Node *n, const std::string &x, int j) {
+        if (!is_lazy(n) || !quad[(size_t)n->col]) return limb(n, x, j);
+        const auto key = std::make_pair(n->col, j >> 2);
+        auto it = wq.find(key);
+        if (it == wq.end()) {
+            std::string v = fresh("q");
+            o << "    const uint4 " << v << " = __ldg(reinterpret_cast<const uint4 *>(g" << n->col << " + (long long)" << (j >> 2)
+              << " * l" << n->col << "));\n";
+            it = wq.emplace(key, v).first;
+        }
+        static const char *f[4] = {".x", ".y", ".z", ".w"};
+        return it->second + f[j & 3];
     }
     // the whole operand as a register array (loads a lazy column)
     std::string whole(const Node *n, const std::string &x) {
         if (!is_lazy(n)) return x;
         std::string t = fresh("t");
         o << "    u32 " << t << "[" << n->L << "];\n#pragma unroll\n    for (int j = 0; j < " << n->L << "; ++j) " << t
-          << "[j] = __ldg(g" << n->col << " + (long long)j * l" << n->col << ");\n";
+          << "[j] = __ldg(g" << n->col << " + " << lazy_off(n->col, -1) << ");\n";
         return t;
+    }
+    // word offset of limb j (-1: the loop variable j) of a lazy column from its row pointer
+    std::string lazy_off(int col, int j) const {
+        const std::string J = j < 0 ? "j" : std::to_string(j), l = "l" + std::to_string(col);
+        if ((size_t)col < quad.size() && quad[(size_t)col])
+            return j < 0 ? "(long long)(j >> 2) * " + l + " + (j & 3)"
+                         : "(long long)" + std::to_string(j >> 2) + " * " + l + " + " + std::to_string(j & 3);
+        return "(long long)" + J + " * " + l;
     }
 
     // constant array of exactly `n` limbs holding v (truncated / zero padded)
@@ -181,12 +208,17 @@ struct Emitter {
                 // top-limb decision (div_top_decide), the full Knuth division only for undecided rows
                 const int E = Lb - T, NAH = La - E;
                 std::string ah = fresh("t"), vh = fresh("t");
+                // the window's limbs (quad columns: their 16-byte loads are emitted here)
+                wq.clear();
+                std::vector<std::string> av, bv;
+                for (int j = 0; j < NAH; ++j) av.push_back(top_limb(L_, a, E + j));
+                for (int j = 0; j < T; ++j) bv.push_back(top_limb(R_, b, E + j));
+                const std::string atop = top_limb(L_, a, La - 1), btop = top_limb(R_, b, Lb - 1);
                 // signs in {0,1} (cond_neg's contract); complement masks 0 - sign
-                o << "    u32 " << t << "[" << L << "], " << na << " = " << limb(L_, a, La - 1) << " >> 31, " << nb
-                  << " = " << limb(R_, b, Lb - 1) << " >> 31;\n";
+                o << "    u32 " << t << "[" << L << "], " << na << " = " << atop << " >> 31, " << nb << " = " << btop << " >> 31;\n";
                 o << "    u32 " << ah << "[" << NAH << "], " << vh << "[" << T << "];\n";
-                for (int j = 0; j < NAH; ++j) o << "    " << ah << "[" << j << "] = " << limb(L_, a, E + j) << " ^ (0u - " << na << ");\n";
-                for (int j = 0; j < T; ++j) o << "    " << vh << "[" << j << "] = " << limb(R_, b, E + j) << " ^ (0u - " << nb << ");\n";
+                for (int j = 0; j < NAH; ++j) o << "    " << ah << "[" << j << "] = " << av[(size_t)j] << " ^ (0u - " << na << ");\n";
+                for (int j = 0; j < T; ++j) o << "    " << vh << "[" << j << "] = " << bv[(size_t)j] << " ^ (0u - " << nb << ");\n";
                 o << "    if (!div_top_decide<" << NAH << "," << T << "," << c.w.size() << "," << L << ">(" << t << ", " << ah << ", " << vh << ", " << kc << ")) {\n";
                 const std::string fa = whole(L_, a), fb = whole(R_, b);
                 o << "    u32 " << ua << "[" << La << "], " << ub << "[" << Lb << "], " << na << "x, " << nb << "x; abs_copy(" << ua << ", " << fa << ", " << na << "x); abs_copy(" << ub << ", " << fb << ", " << nb << "x);\n";
@@ -241,8 +273,11 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
         std::vector<int> uses(cols.size(), 0), div_uses(cols.size(), 0);
         div_only_uses(root, uses, div_uses);
         E.lazy.assign(cols.size(), false);
-        for (size_t c = 0; c < cols.size(); ++c)
+        E.quad.assign(cols.size(), false);
+        for (size_t c = 0; c < cols.size(); ++c) {
             E.lazy[c] = used[c] && cols[c].Lb == 0 && uses[c] > 0 && uses[c] == div_uses[c];
+            E.quad[c] = cols[c].Q;
+        }
     }
     std::string res = E.emit(root);
 
@@ -382,6 +417,11 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
         if (!used[c] || E.lazy[c] || cols[c].Lb > 0) continue;
         const int Lc = cols[c].limbs;
         k << "        u32 x" << c << "[R][" << Lc << "] = {};\n";
+        if (cols[c].Q) {   // limb quads: one 16-byte load per quad and row
+            k << "        if (live) { const uint4 *q = reinterpret_cast<const uint4 *>(P.col[" << c << "]) + base; const long long ld = P.ld[" << c << "];\n";
+            k << "#pragma unroll\n          for (int r = 0; r < R; ++r) ld_quads<" << Lc << "," << (R == 1 ? "true" : "false") << ">(x" << c << "[r], q + r, ld); }\n";
+            continue;
+        }
         k << "        if (live) { const u32 *p = P.col[" << c << "] + base; const long long ld = P.ld[" << c << "];\n";
         if (R == 4) {
             k << "#pragma unroll\n          for (int j = 0; j < " << Lc << "; ++j) { const uint4 v = __ldcs(reinterpret_cast<const uint4 *>(p + j * ld));"
@@ -398,7 +438,8 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     first = true;
     for (size_t c = 0; c < cols.size(); ++c) {
         if (!used[c]) continue;
-        if (E.lazy[c]) k << (first ? "" : ", ") << "P.col[" << c << "] + base + r, P.ld[" << c << "]";
+        if (E.lazy[c] && cols[c].Q) k << (first ? "" : ", ") << "P.col[" << c << "] + 4 * (base + r), 4 * P.ld[" << c << "]";
+        else if (E.lazy[c]) k << (first ? "" : ", ") << "P.col[" << c << "] + base + r, P.ld[" << c << "]";
         else k << (first ? "" : ", ") << "x" << c << "[r]";
         first = false;
     }

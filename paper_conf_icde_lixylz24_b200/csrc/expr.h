@@ -20,8 +20,9 @@ struct Node {
 };
 
 // Lb > 0: the column is stored in the compact byte layout (the paper's
-// cDecimal): Lb bytes per row, row-major; else limb planes
-struct ColType { int p, s, limbs; int Lb = 0; };
+// cDecimal): Lb bytes per row, row-major; Q: limb quads (up.h
+// UP_LAYOUT_QUADS); else limb planes
+struct ColType { int p, s, limbs; int Lb = 0; bool Q = false; };
 
 // Parse "c1*c2 - c3/c4" (SQL precedence, left-assoc, unary -, parentheses,
 // literals typed by value: 1.23 -> DECIMAL(3,2), 10 -> DECIMAL(2,0),

@@ -56,6 +56,43 @@ __global__ void __launch_bounds__(256) k_to_bin(const u32 *__restrict__ planes, 
     }
 }
 
+// limb planes -> limb quads (up.h UP_LAYOUT_QUADS): quad g of row i =
+// limbs 4g..4g+3 as one uint4 at q[g*ldq + i]; limb L = the sign flag (1 for a
+// negative row), the limbs above it 0.  One thread per (row, quad): 16-byte
+// stores coalesced across the warp.
+__global__ void __launch_bounds__(256) k_planes_to_quads(const u32 *__restrict__ planes, int L, long long ld,
+                                                         long long n, uint4 *__restrict__ q, long long ldq) {
+    const int G = (L + 1 + 3) / 4;
+    const long long total = n * G, stride = (long long)gridDim.x * blockDim.x;
+    for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
+        const long long i = t % n;
+        const int g = (int)(t / n);
+        u32 w[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const int j = 4 * g + k;
+            w[k] = j < L ? planes[(long long)j * ld + i] : j == L ? planes[(long long)(L - 1) * ld + i] >> 31 : 0u;
+        }
+        q[(long long)g * ldq + i] = make_uint4(w[0], w[1], w[2], w[3]);
+    }
+}
+
+// limb quads -> limb planes (the flag and padding limbs are dropped)
+__global__ void __launch_bounds__(256) k_quads_to_planes(const uint4 *__restrict__ q, long long ldq, int L, long long n,
+                                                         u32 *__restrict__ planes, long long ld) {
+    const int G = (L + 3) / 4;   // quads holding value limbs
+    const long long total = n * G, stride = (long long)gridDim.x * blockDim.x;
+    for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
+        const long long i = t % n;
+        const int g = (int)(t / n);
+        const uint4 v = q[(long long)g * ldq + i];
+        const u32 w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+            if (4 * g + k < L) planes[(long long)(4 * g + k) * ld + i] = w[k];
+    }
+}
+
 // out = sum of nranks la-limb two's-complement partials, mod 2^(32 la), in
 // rank order (exact; order only matters for readability -- integer sums
 // commute).  One block: limb-parallel 64-bit column sums, then one carry pass.
@@ -336,6 +373,18 @@ cudaError_t upk_launch_from_compact(const uint8_t *bytes, int Lb, long long n, c
 cudaError_t upk_launch_to_compact(const uint32_t *planes, int L, long long ld, long long n, uint8_t *bytes, int Lb,
                                  cudaStream_t st) {
     k_to_compact<<<grid_for(n, 256), 256, 0, st>>>(planes, L, ld, n, bytes, Lb);
+    return cudaGetLastError();
+}
+
+cudaError_t upk_launch_planes_to_quads(const uint32_t *planes, int L, long long ld, long long n, uint32_t *quads,
+                                      long long ldq, cudaStream_t st) {
+    k_planes_to_quads<<<grid_for(n * ((L + 4) / 4), 256), 256, 0, st>>>(planes, L, ld, n, (uint4 *)quads, ldq);
+    return cudaGetLastError();
+}
+
+cudaError_t upk_launch_quads_to_planes(const uint32_t *quads, long long ldq, int L, long long n, uint32_t *planes,
+                                      long long ld, cudaStream_t st) {
+    k_quads_to_planes<<<grid_for(n * ((L + 3) / 4), 256), 256, 0, st>>>((const uint4 *)quads, ldq, L, n, planes, ld);
     return cudaGetLastError();
 }
 

@@ -50,6 +50,13 @@ cudaError_t upk_launch_from_compact(const uint8_t *bytes, int Lb, long long n, c
                                    uint32_t *out, long long ld, uint32_t *flags, cudaStream_t st);
 cudaError_t upk_launch_to_compact(const uint32_t *planes, int L, long long ld, long long n, uint8_t *bytes, int Lb,
                                  cudaStream_t st);
+cudaError_t upk_launch_planes_to_quads(const uint32_t *planes, int L, long long ld, long long n, uint32_t *quads,
+                                      long long ldq, cudaStream_t st);
+cudaError_t upk_launch_quads_to_planes(const uint32_t *quads, long long ldq, int L, long long n, uint32_t *planes,
+                                      long long ld, cudaStream_t st);
+cudaError_t upk_launch_contract_tq(const uint32_t *A, long long lda, int La, const uint32_t *B, long long ldb, int Lb,
+                                   long long n, int sign, unsigned long long *ws, uint32_t *ticket, uint32_t *result,
+                                   int LA, int num_sms, cudaStream_t st);
 }
 
 namespace {
@@ -134,6 +141,7 @@ struct JitKernel {
     int dyn_smem = 0;      // dynamic shared memory per block (bytes)
     int rows_per_block = 0;  // > 0: warp-per-row kernels (rows per block-iteration)
     bool pdl = false;        // may be launched with programmatic stream serialization
+    bool carveout_max = false;   // preferred shared-memory carveout set to 100 %
     std::string src;
 };
 
@@ -169,6 +177,12 @@ struct up_ctx {
     uint64_t launches = 0;
     double jit_ms = 0.0;
     bool pipelined = false;   // up_set_pipelined: PDL launches of the fused SUM kernels
+    // split SUMs over quad columns: the tensor-core contraction runs on a side
+    // stream (own workspace + ticket) concurrently with the rest kernel
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    unsigned long long *d_ws2 = nullptr;
+    uint32_t *d_ticket2 = nullptr;
     std::mutex mu;
 };
 
@@ -205,7 +219,7 @@ up_status check_column(const up_column *col, const char *what) {
     if (col->p < 1 || col->s < 0) return fail(UP_E_INVAL, "%s: bad DECIMAL(%d,%d)", what, col->p, col->s);
     if (col->limbs != limbs_for_precision(col->p))
         return fail(UP_E_INVAL, "%s: limbs %d != up_limbs(%d) = %d", what, col->limbs, col->p, limbs_for_precision(col->p));
-    if (col->layout != UP_LAYOUT_PLANES && col->layout != UP_LAYOUT_COMPACT)
+    if (col->layout != UP_LAYOUT_PLANES && col->layout != UP_LAYOUT_COMPACT && col->layout != UP_LAYOUT_QUADS)
         return fail(UP_E_INVAL, "%s: unknown layout %d", what, col->layout);
     if (col->layout == UP_LAYOUT_COMPACT) {
         if (col->ld != up_compact_bytes(col->p))
@@ -222,8 +236,8 @@ up_status check_column(const up_column *col, const char *what) {
 }
 
 up_status need_planes(const up_column *col, const char *what) {
-    if (col && col->layout == UP_LAYOUT_COMPACT)
-        return fail(UP_E_UNSUPPORTED, "%s: this call needs a limb-plane column (compact columns: up_eval_expr / "
+    if (col && col->layout != UP_LAYOUT_PLANES)
+        return fail(UP_E_UNSUPPORTED, "%s: this call needs a limb-plane column (compact and quad columns: up_eval_expr / "
                                       "up_sum_expr / up_filter)", what);
     return UP_OK;
 }
@@ -339,7 +353,8 @@ up_status type_expr(const char *expr, const up_column *cols, int ncols, Typed &t
         if (cols[i].p < 1 || cols[i].s < 0 || cols[i].limbs != limbs_for_precision(cols[i].p))
             return fail(UP_E_INVAL, "column %d: bad type/limbs", i + 1);
         t.types.push_back({cols[i].p, cols[i].s, cols[i].limbs,
-                           cols[i].layout == UP_LAYOUT_COMPACT ? up_compact_bytes(cols[i].p) : 0});
+                           cols[i].layout == UP_LAYOUT_COMPACT ? up_compact_bytes(cols[i].p) : 0,
+                           cols[i].layout == UP_LAYOUT_QUADS});
     }
     std::string err;
     t.root = parse_expr(expr, ncols, err);
@@ -353,7 +368,8 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     k += '|';
     k += expr;
     for (int i = 0; i < ncols; ++i)
-        k += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s) + (cols[i].layout == UP_LAYOUT_COMPACT ? "c" : "");
+        k += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s) +
+             (cols[i].layout == UP_LAYOUT_COMPACT ? "c" : cols[i].layout == UP_LAYOUT_QUADS ? "q" : "");
     k += "|" + std::to_string(extra);
     if (getenv("UP_NO_OPT")) k += "|noopt";
     if (getenv("UP_NO_WIDE")) k += "|nowide";
@@ -361,10 +377,17 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     return k;
 }
 
-up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream_t st) {
+// bps_leave: resident blocks per SM left free for a concurrent kernel
+up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream_t st, int bps_leave = 0) {
     long long per_block = k->rows_per_block > 0 ? k->rows_per_block : (long long)k->threads * k->rows_per_thread;
     long long want = (n + per_block - 1) / per_block;
-    long long cap = (long long)k->blocks_per_sm * c->num_sms;
+    long long cap = (long long)std::max(1, k->blocks_per_sm - bps_leave) * c->num_sms;
+    if (bps_leave > 0 && !k->carveout_max) {
+        // blocks of kernels with different shared-memory carveouts cannot share an
+        // SM: the concurrent kernel (the tensor-core contraction) needs ~200 KB
+        CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100));
+        k->carveout_max = true;
+    }
     int grid = (int)std::max(1ll, std::min(want, cap));
     void *args[] = {&P};
     if (k->pdl && c->pipelined) {
@@ -408,7 +431,7 @@ up_status expr_kernel(up_ctx *c, const char *expr, const up_column *cols, int nc
     const Node *gen_root = opt_root ? opt_root.get() : t.root.get();
     // wide SUM regime: warp per row, linear decomposition into summed terms
     bool any_compact = false;
-    for (const ColType &ct : t.types) any_compact = any_compact || ct.Lb > 0;
+    for (const ColType &ct : t.types) any_compact = any_compact || ct.Lb > 0 || ct.Q;   // wide regime reads planes
     if (sum && !any_compact && max_limbs(gen_root) >= kWideMinLimbs && LA <= 512 && !getenv("UP_NO_WIDE"))
         src = gen_wide_sum_kernel(gen_root, t.types, LA, info);
     if (src.empty()) {
@@ -484,6 +507,7 @@ extern "C" {
 const char *up_last_error(void) { return g_err.c_str(); }
 
 int32_t up_limbs(int32_t p) { return limbs_for_precision(p); }
+int32_t up_quads(int32_t p) { return (limbs_for_precision(p) + 1 + 3) / 4; }
 int64_t up_ld(int64_t n) { return (n + 3) & ~3ll; }
 int32_t up_sum_precision(int32_t p, int64_t n_global) { return sum_precision(p, n_global); }
 
@@ -519,6 +543,11 @@ up_status up_ctx_destroy(up_ctx *c) {
     for (auto &kv : c->pow10_dev) cudaFree(kv.second);
     cudaFree(c->d_ws);
     cudaFree(c->d_ticket);
+    if (c->d_ws2) cudaFree(c->d_ws2);
+    if (c->d_ticket2) cudaFree(c->d_ticket2);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
+    if (c->side) cudaStreamDestroy(c->side);
     cudaFree(c->d_flags);
     if (c->d_stage) cudaFree(c->d_stage);
     if (c->d_scratch) cudaFree(c->d_scratch);
@@ -545,6 +574,15 @@ up_status up_column_from_device_bin(up_ctx *c, const uint32_t *d_mag, int32_t W,
         if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)dst->limbs * (size_t)ld, (void **)&planes)) return s;
         CUDA_TRY(upk_launch_from_bin(d_mag, W, d_neg, dst->n, bound, dst->limbs, planes, ld, c->d_flags, (cudaStream_t)stream));
         CUDA_TRY(upk_launch_to_compact(planes, dst->limbs, ld, dst->n, (uint8_t *)dst->data, (int)dst->ld, (cudaStream_t)stream));
+        c->launches += 2;
+        return UP_OK;
+    }
+    if (dst->layout == UP_LAYOUT_QUADS) {   // via limb planes in the ctx scratch
+        const long long ld = (dst->n + 3) & ~3ll;
+        uint32_t *planes = nullptr;
+        if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)dst->limbs * (size_t)ld, (void **)&planes)) return s;
+        CUDA_TRY(upk_launch_from_bin(d_mag, W, d_neg, dst->n, bound, dst->limbs, planes, ld, c->d_flags, (cudaStream_t)stream));
+        CUDA_TRY(upk_launch_planes_to_quads(planes, dst->limbs, ld, dst->n, dst->data, dst->ld, (cudaStream_t)stream));
         c->launches += 2;
         return UP_OK;
     }
@@ -634,6 +672,16 @@ up_status up_column_from_device_compact(up_ctx *c, const uint8_t *d_bytes, up_co
         c->launches++;
         return UP_OK;
     }
+    if (dst->layout == UP_LAYOUT_QUADS) {   // via limb planes in the ctx scratch
+        const long long ld = (dst->n + 3) & ~3ll;
+        uint32_t *planes = nullptr;
+        if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)dst->limbs * (size_t)ld, (void **)&planes)) return s;
+        CUDA_TRY(upk_launch_from_compact(d_bytes, up_compact_bytes(dst->p), dst->n, bound, dst->limbs, planes, ld,
+                                         c->d_flags, (cudaStream_t)stream));
+        CUDA_TRY(upk_launch_planes_to_quads(planes, dst->limbs, ld, dst->n, dst->data, dst->ld, (cudaStream_t)stream));
+        c->launches += 2;
+        return UP_OK;
+    }
     CUDA_TRY(upk_launch_from_compact(d_bytes, up_compact_bytes(dst->p), dst->n, bound, dst->limbs, dst->data, dst->ld,
                                      c->d_flags, (cudaStream_t)stream));
     c->launches++;
@@ -676,7 +724,17 @@ up_status up_column_to_host_compact(up_ctx *c, const up_column *col, uint8_t *by
     }
     std::lock_guard<std::mutex> g(c->mu);
     if (up_status s = ensure_stage(c, nb, st)) return s;
-    CUDA_TRY(upk_launch_to_compact(col->data, col->limbs, col->ld, col->n, (uint8_t *)c->d_stage, Lb, st));
+    const uint32_t *planes = col->data;
+    long long ld = col->ld;
+    if (col->layout == UP_LAYOUT_QUADS) {   // quads -> limb planes in the ctx scratch first
+        ld = (col->n + 3) & ~3ll;
+        uint32_t *pl = nullptr;
+        if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)col->limbs * (size_t)ld, (void **)&pl)) return s;
+        CUDA_TRY(upk_launch_quads_to_planes(col->data, col->ld, col->limbs, col->n, pl, ld, st));
+        c->launches++;
+        planes = pl;
+    }
+    CUDA_TRY(upk_launch_to_compact(planes, col->limbs, ld, col->n, (uint8_t *)c->d_stage, Lb, st));
     c->launches++;
     CUDA_TRY(cudaMemcpyAsync(bytes, c->d_stage, nb, cudaMemcpyDeviceToHost, st));
     CUDA_TRY(cudaStreamSynchronize(st));
@@ -704,6 +762,13 @@ up_status up_column_to_host_bin(up_ctx *c, const up_column *col, uint32_t *mag, 
         if (up_status s = pow10_device(c, col->p, &bound)) return s;
         CUDA_TRY(upk_launch_from_compact((const uint8_t *)col->data, (int)col->ld, col->n, bound, col->limbs, pl, ld,
                                          c->d_flags, st));
+        c->launches++;
+        planes = pl;
+    } else if (col->layout == UP_LAYOUT_QUADS) {   // quads -> limb planes in the ctx scratch first
+        ld = (col->n + 3) & ~3ll;
+        uint32_t *pl = nullptr;
+        if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)col->limbs * (size_t)ld, (void **)&pl)) return s;
+        CUDA_TRY(upk_launch_quads_to_planes(col->data, col->ld, col->limbs, col->n, pl, ld, st));
         c->launches++;
         planes = pl;
     }
@@ -744,6 +809,7 @@ up_status up_eval_expr(up_ctx *c, const char *expr, const up_column *cols, int n
         if (cols[i].n != cols[0].n) return fail(UP_E_INVAL, "columns differ in length");
     }
     if (up_status s = check_column(out, "out")) return s;
+    if (out->layout != UP_LAYOUT_PLANES) return fail(UP_E_UNSUPPORTED, "out must be limb planes");
     std::lock_guard<std::mutex> g(c->mu);
     JitKernel *k = nullptr;
     Node *root = nullptr;
@@ -851,7 +917,12 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
                 for (const SplitTerm &st : pl.prods) {
                     const int La = cols[st.col_a].limbs, Lb = cols[st.col_b].limbs;
                     JitKernel *kc = nullptr;
-                    if (!(use_tc && upk_contract_tc_slots(La, Lb) <= kWsSlots)) {
+                    const bool qa = cols[st.col_a].layout == UP_LAYOUT_QUADS, qb = cols[st.col_b].layout == UP_LAYOUT_QUADS;
+                    const bool tc_ok = use_tc && upk_contract_tc_slots(La, Lb) <= kWsSlots;
+                    // quad columns: the tensor-core contraction reads both operands as quads;
+                    // otherwise the whole SUM stays in the fused kernel
+                    if ((qa || qb) && !(qa && qb && tc_ok)) { pl.split = false; break; }
+                    if (!tc_ok) {
                         std::string key = "contract|" + std::to_string(La) + "|" + std::to_string(Lb) + "|" + std::to_string(LAs) +
                                           "|" + std::to_string(st.sign) + "|" + std::to_string(st.col_a) + "|" + std::to_string(st.col_b);
                         if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
@@ -860,9 +931,10 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
                     }
                     pl.cc_kernels.push_back(kc);   // nullptr: tensor-core contraction
                 }
-                if (rest) {
+                if (pl.split && rest) {
                     std::string key = "rest|" + canonical(rest.get()) + "|" + std::to_string(LAs);
-                    for (int i = 0; i < ncols; ++i) key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s);
+                    for (int i = 0; i < ncols; ++i)
+                        key += "|" + std::to_string(cols[i].p) + "," + std::to_string(cols[i].s) + "," + std::to_string(cols[i].layout);
                     Node *rr = rest.get();
                     if (up_status s = kernel_for(c, key, [&](GenInfo &info) {
                             GenOpts o;
@@ -880,7 +952,11 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             const int T = (int)pl.prods.size() + (pl.rest_kernel ? 1 : 0);
             const size_t need = (size_t)T * (size_t)LAs;
             if (need > c->parts_words) {
-                if (c->d_parts) { CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream)); CUDA_TRY(cudaFree(c->d_parts)); }
+                if (c->d_parts) {
+                    CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream));
+                    if (c->side) CUDA_TRY(cudaStreamSynchronize(c->side));
+                    CUDA_TRY(cudaFree(c->d_parts));
+                }
                 CUDA_TRY(cudaMalloc(&c->d_parts, sizeof(uint32_t) * need * 2));
                 c->parts_words = need * 2;
             }
@@ -889,14 +965,40 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             P.ws = c->d_ws;
             P.ticket = c->d_ticket;
             P.flags = c->d_flags;
+            // quad columns: the tensor-core contraction (a few warps and the
+            // shared-memory stages, HBM-bound) runs on the side stream while the
+            // integer-bound rest kernel fills the SMs' remaining block slots on
+            // the caller's stream; joined before the combine (UP_SERIAL_SPLIT:
+            // one stream, back to back)
+            bool overlap = pl.rest_kernel != nullptr && !getenv("UP_SERIAL_SPLIT");
+            for (size_t q = 0; q < pl.prods.size() && overlap; ++q)
+                overlap = !pl.cc_kernels[q] && cols[pl.prods[q].col_a].layout == UP_LAYOUT_QUADS;
+            cudaStream_t tcs = (cudaStream_t)stream;
+            unsigned long long *tws = c->d_ws;
+            uint32_t *ttk = c->d_ticket;
+            if (overlap) {
+                if (!c->side) {
+                    CUDA_TRY(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
+                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+                    CUDA_TRY(cudaMalloc(&c->d_ws2, sizeof(unsigned long long) * 2 * 1024));
+                    CUDA_TRY(cudaMemset(c->d_ws2, 0, sizeof(unsigned long long) * 2 * 1024));
+                    CUDA_TRY(cudaMalloc(&c->d_ticket2, 64));
+                    CUDA_TRY(cudaMemset(c->d_ticket2, 0, 64));
+                    CUDA_TRY(cudaDeviceSynchronize());
+                }
+                CUDA_TRY(cudaEventRecord(c->ev_fork, (cudaStream_t)stream));
+                CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+                tcs = c->side; tws = c->d_ws2; ttk = c->d_ticket2;
+            }
             int ti = 0;
             for (size_t q = 0; q < pl.prods.size(); ++q) {
                 const SplitTerm &st = pl.prods[q];
                 const up_column &ca = cols[st.col_a], &cb = cols[st.col_b];
                 if (!pl.cc_kernels[q]) {
-                    CUDA_TRY(upk_launch_contract_tc(ca.data, ca.ld, ca.limbs, cb.data, cb.ld, cb.limbs, cols[0].n, st.sign,
-                                                    c->d_ws, c->d_ticket, c->d_parts + (size_t)ti++ * LAs, LAs, c->num_sms,
-                                                    (cudaStream_t)stream));
+                    auto tc = ca.layout == UP_LAYOUT_QUADS ? upk_launch_contract_tq : upk_launch_contract_tc;
+                    CUDA_TRY(tc(ca.data, ca.ld, ca.limbs, cb.data, cb.ld, cb.limbs, cols[0].n, st.sign, tws, ttk,
+                                c->d_parts + (size_t)ti++ * LAs, LAs, c->num_sms, tcs));
                     c->launches++;
                     continue;
                 }
@@ -905,7 +1007,12 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             }
             if (pl.rest_kernel) {
                 P.result = c->d_parts + (size_t)ti++ * LAs;
-                if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream)) return s;
+                // one block slot per SM left to the contraction CTA
+                if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream, overlap ? 1 : 0)) return s;
+            }
+            if (overlap) {
+                CUDA_TRY(cudaEventRecord(c->ev_join, c->side));
+                CUDA_TRY(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_join, 0));
             }
             if (pl.rest_kernel && pl.rest_scale > 0) {
                 const uint32_t *d_sc = nullptr;
@@ -1068,8 +1175,10 @@ up_status up_eval_tpi(up_ctx *c, const char *op, const up_column *a, const up_co
     if (o < 0) return fail(UP_E_INVAL, "operator must be + - * /");
     if (div_algo != 0 && div_algo != 1) return fail(UP_E_INVAL, "div_algo must be 0 (long division) or 1 (Newton-Raphson)");
     const up_column cols[2] = {*a, *b};
-    for (int i = 0; i < 2; ++i)
+    for (int i = 0; i < 2; ++i) {
         if (up_status s = check_column(&cols[i], "input")) return s;
+        if (cols[i].layout == UP_LAYOUT_QUADS) return fail(UP_E_UNSUPPORTED, "tpi inputs: limb planes or compact rows");
+    }
     if (a->n != b->n) return fail(UP_E_INVAL, "columns differ in length");
     if (up_status s = check_column(out, "out")) return s;
     if (out->layout != UP_LAYOUT_PLANES) return fail(UP_E_UNSUPPORTED, "out must be limb planes");

@@ -32,7 +32,7 @@ class up_column(ctypes.Structure):
 
 
 _lib = None
-EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_ld", "up_sum_precision",
+EXPORTS = ["up_last_error", "up_ctx_create", "up_ctx_destroy", "up_limbs", "up_quads", "up_ld", "up_sum_precision",
            "up_column_from_host_bin", "up_column_from_device_bin", "up_column_from_host",
            "up_column_to_host_bin", "up_expr_type", "up_eval_expr", "up_sum_type", "up_sum_expr",
            "up_sum", "up_sum_combine", "up_modexp", "up_modexp_sum_type", "up_modexp_sum",
@@ -60,6 +60,7 @@ def lib():
     L.up_last_error.restype = c.c_char_p
     L.up_limbs.argtypes = [c.c_int32]; L.up_limbs.restype = c.c_int32
     L.up_ld.argtypes = [c.c_int64]; L.up_ld.restype = c.c_int64
+    L.up_quads.argtypes = [c.c_int32]; L.up_quads.restype = c.c_int32
     L.up_sum_precision.argtypes = [c.c_int32, c.c_int64]; L.up_sum_precision.restype = c.c_int32
     L.up_ctx_create.argtypes = [c.c_int, c.POINTER(P)]
     L.up_ctx_destroy.argtypes = [P]
@@ -124,6 +125,10 @@ def compact_bytes(p: int) -> int:
     return lib().up_compact_bytes(p)
 
 
+def quads(p: int) -> int:
+    return lib().up_quads(p)
+
+
 def ld_for(n: int) -> int:
     return lib().up_ld(n)
 
@@ -141,24 +146,31 @@ def _stream_ptr(stream) -> Optional[int]:
     return stream.cuda_stream
 
 
-LAYOUT_PLANES, LAYOUT_COMPACT = 0, 1
+LAYOUT_PLANES, LAYOUT_COMPACT, LAYOUT_QUADS = 0, 1, 2
+_LAYOUTS = {"planes": LAYOUT_PLANES, "compact": LAYOUT_COMPACT, "quads": LAYOUT_QUADS}
 
 
 class Column:
     """A DECIMAL(p,s) column on the GPU.  layout "planes": `limbs`
     two's-complement limb planes in a torch int32 tensor (limbs, ld);
     layout "compact": the paper's compact byte rows (Lb = compact_bytes(p)
-    bytes per row, up.h UP_LAYOUT_COMPACT) in a uint8 tensor padded to 16 bytes."""
+    bytes per row, up.h UP_LAYOUT_COMPACT) in a uint8 tensor padded to 16 bytes;
+    layout "quads": limb quads (up.h UP_LAYOUT_QUADS), an int32 tensor
+    (quads(p), ld, 4)."""
 
     def __init__(self, p: int, s: int, n: int, device="cuda", data=None, layout: str = "planes"):
         import torch
         self.p, self.s, self.n = p, s, n
         self.limbs = limbs(p)
-        self.layout = LAYOUT_COMPACT if layout == "compact" else LAYOUT_PLANES
+        self.layout = _LAYOUTS[layout]
         if self.layout == LAYOUT_COMPACT:
             self.ld = compact_bytes(p)
             if data is None:
                 data = torch.empty(((n * self.ld + 15) // 16) * 16 + 16, dtype=torch.uint8, device=device)
+        elif self.layout == LAYOUT_QUADS:
+            self.ld = ld_for(n)
+            if data is None:
+                data = torch.empty((quads(p), max(self.ld, 4), 4), dtype=torch.int32, device=device)
         else:
             self.ld = ld_for(n)
             if data is None:
@@ -551,12 +563,16 @@ def result_to_string(limb_tensor, s: int) -> str:
 
 # ---------------------------------------------------------------------- diagnostics
 def gen_source(variant: str, expr: str, types: Sequence[tuple], n_global: int = 1,
-               compact: Optional[Sequence[bool]] = None) -> str:
-    """Generated kernel source (no GPU); compact[i]: column i in the compact layout."""
+               compact: Optional[Sequence[bool]] = None, layouts: Optional[Sequence[str]] = None) -> str:
+    """Generated kernel source (no GPU); compact[i]: column i in the compact
+    layout; layouts[i]: "planes" / "compact" / "quads"."""
     arr = (up_column * max(1, len(types)))()
     for i, (p, s) in enumerate(types):
-        if compact and compact[i]:
+        lay = layouts[i] if layouts else ("compact" if compact and compact[i] else "planes")
+        if lay == "compact":
             arr[i] = up_column(n_global, compact_bytes(p), p, s, limbs(p), LAYOUT_COMPACT, None)
+        elif lay == "quads":
+            arr[i] = up_column(n_global, ld_for(n_global), p, s, limbs(p), LAYOUT_QUADS, None)
         else:
             arr[i] = up_column(n_global, ld_for(n_global), p, s, limbs(p), 0, None)
     buf = ctypes.create_string_buffer(1 << 24)
