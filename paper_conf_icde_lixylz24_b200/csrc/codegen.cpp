@@ -72,6 +72,7 @@ void div_only_uses(const Node *n, std::vector<int> &uses, std::vector<int> &div_
 
 struct Emitter {
     std::ostringstream o;
+    std::ostringstream pre;   // out-of-line helpers, emitted before eval_row
     int tmp = 0;
     std::vector<bool> lazy;   // column c is read from global memory by the divisions that use it
     std::vector<bool> quad;   // column c is stored as limb quads (limb j at g + (j>>2)*l + (j&3))
@@ -220,6 +221,34 @@ struct Emitter {
                 for (int j = 0; j < NAH; ++j) o << "    " << ah << "[" << j << "] = " << av[(size_t)j] << " ^ (0u - " << na << ");\n";
                 for (int j = 0; j < T; ++j) o << "    " << vh << "[" << j << "] = " << bv[(size_t)j] << " ^ (0u - " << nb << ");\n";
                 o << "    if (!div_top_decide<" << NAH << "," << T << "," << c.w.size() << "," << L << ">(" << t << ", " << ah << ", " << vh << ", " << kc << ")) {\n";
+                if (is_lazy(L_) && is_lazy(R_)) {
+                    // both operands are columns: the (rare) full division runs out
+                    // of line, so its wide arrays do not share the row loop's registers
+                    const std::string fn = fresh("divfb"), rt = fn + "_r";
+                    const int la = L_->col, lb = R_->col;
+                    auto ld = [&](int col, const char *g, const char *l) {
+                        const bool qd = quad[(size_t)col];
+                        return std::string("__ldg(") + g + " + " + (qd ? std::string("(long long)(j >> 2) * ") + l + " + (j & 3)" : std::string("(long long)j * ") + l) + ")";
+                    };
+                    pre << "struct " << rt << " { u32 w[" << L << "]; u32 fl; };\n";
+                    pre << "__device__ __noinline__ " << rt << " " << fn << "(const u32 *__restrict__ ga, long long la, const u32 *__restrict__ gb, long long lb) {\n";
+                    pre << "    const u32 kc[" << c.w.size() << "] = " << limbs_init(std::vector<uint32_t>(c.w.begin(), c.w.end())) << ";\n";
+                    pre << "    u32 fa[" << La << "], fb[" << Lb << "];\n";
+                    pre << "#pragma unroll\n    for (int j = 0; j < " << La << "; ++j) fa[j] = " << ld(la, "ga", "la") << ";\n";
+                    pre << "#pragma unroll\n    for (int j = 0; j < " << Lb << "; ++j) fb[j] = " << ld(lb, "gb", "lb") << ";\n";
+                    pre << "    u32 ua[" << La << "], ub[" << Lb << "], na, nb; abs_copy(ua, fa, na); abs_copy(ub, fb, nb);\n";
+                    pre << "    u32 uu[" << NU << "]; mul_mag<" << La << "," << c.w.size() << "," << NU << ">(uu, ua, kc);\n";
+                    pre << "    u32 rr[" << Lb << "]; " << rt << " r;\n";
+                    pre << "    r.fl = divmod_mag<" << NU << "," << Lb << "," << L << ",false>(r.w, rr, uu, ub);\n";
+                    pre << "    return r;\n}\n\n";
+                    o << "    { const " << rt << " r = " << fn << "(g" << la << ", l" << la << ", g" << lb << ", l" << lb << "); fl |= r.fl;\n";
+                    o << "#pragma unroll\n      for (int j = 0; j < " << L << "; ++j) " << t << "[j] = r.w[j]; }\n";
+                    o << "    }\n";
+                    std::string kb = konst(HBig::pow10(n->p), L);
+                    o << "    if (!lt(" << t << ", " << kb << ")) fl |= F_OVERFLOW;\n";
+                    o << "    cond_neg(" << t << ", " << na << " ^ " << nb << ");\n";
+                    return t;
+                }
                 const std::string fa = whole(L_, a), fb = whole(R_, b);
                 o << "    u32 " << ua << "[" << La << "], " << ub << "[" << Lb << "], " << na << "x, " << nb << "x; abs_copy(" << ua << ", " << fa << ", " << na << "x); abs_copy(" << ub << ", " << fb << ", " << nb << "x);\n";
                 o << "    u32 " << uu << "[" << NU << "]; mul_mag<" << La << "," << c.w.size() << "," << NU << ">(" << uu << ", " << ua << ", " << kc << ");\n";
@@ -285,6 +314,7 @@ std::string gen_expr_kernel(const Node *root, const std::vector<ColType> &cols, 
     k << "// generated by libup codegen: " << canonical(root) << "  type (" << root->p << "," << root->s << ") L=" << LOUT << "\n";
     k << mul_variant_define() << "#include \"up_dev.cuh\"\n#include \"up_kparams.h\"\nusing namespace up;\n\n";
     // per-row evaluation with everything in registers
+    k << E.pre.str();
     k << "__device__ __forceinline__ void eval_row(";
     bool first = true;
     for (size_t c = 0; c < cols.size(); ++c) {
