@@ -490,8 +490,10 @@ def main():
     ap.add_argument("--rows", type=int, default=0, help="rows per GPU (default: the config's)")
     ap.add_argument("--global-rows", type=int, default=0, help="total rows, sharded over the GPUs (strong scaling)")
     ap.add_argument("--impl", default="up", choices=["up", "reference"])
-    ap.add_argument("--layout", default="planes", choices=["planes", "compact", "quads"],
-                    help="column storage for the expression configs (1-3): limb planes or the paper's compact rows")
+    ap.add_argument("--layout", default=None, choices=["planes", "compact", "quads"],
+                    help="column storage for the expression configs (1-3): limb planes, the paper's compact rows or "
+                         "limb quads (default: planes for 1-2, quads for 3 -- the layout its tensor-core "
+                         "contraction reads straight from TMA)")
     ap.add_argument("--ref-rows", type=int, default=200_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-pipelined", action="store_true",
@@ -516,6 +518,8 @@ def main():
         s = {200: 50, 500: 75, 1000: 100}.get(args.p, args.p // 4)
         cfg["types"] = [(args.p, s)] * 4
         cfg["name"] = f"cfg3 SUM(c1*c2 - c3/c4) DECIMAL({args.p},{s})"
+    if args.layout is None:
+        args.layout = "quads" if cfg["kind"] == "expr" and cfg["types"][0][0] >= 100 else "planes"
     if not args.steps:
         args.steps = {"expr": 200, "modexp": 5, "sin": 3}[cfg["kind"]] if cfg["kind"] != "expr" or \
             cfg["types"][0][0] < 100 else 5

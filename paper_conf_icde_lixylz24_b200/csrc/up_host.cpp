@@ -141,7 +141,6 @@ struct JitKernel {
     int dyn_smem = 0;      // dynamic shared memory per block (bytes)
     int rows_per_block = 0;  // > 0: warp-per-row kernels (rows per block-iteration)
     bool pdl = false;        // may be launched with programmatic stream serialization
-    bool carveout_max = false;   // preferred shared-memory carveout set to 100 %
     std::string src;
 };
 
@@ -177,12 +176,6 @@ struct up_ctx {
     uint64_t launches = 0;
     double jit_ms = 0.0;
     bool pipelined = false;   // up_set_pipelined: PDL launches of the fused SUM kernels
-    // split SUMs over quad columns: the tensor-core contraction runs on a side
-    // stream (own workspace + ticket) concurrently with the rest kernel
-    cudaStream_t side = nullptr;
-    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
-    unsigned long long *d_ws2 = nullptr;
-    uint32_t *d_ticket2 = nullptr;
     std::mutex mu;
 };
 
@@ -377,17 +370,10 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     return k;
 }
 
-// bps_leave: resident blocks per SM left free for a concurrent kernel
-up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream_t st, int bps_leave = 0) {
+up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream_t st) {
     long long per_block = k->rows_per_block > 0 ? k->rows_per_block : (long long)k->threads * k->rows_per_thread;
     long long want = (n + per_block - 1) / per_block;
-    long long cap = (long long)std::max(1, k->blocks_per_sm - bps_leave) * c->num_sms;
-    if (bps_leave > 0 && !k->carveout_max) {
-        // blocks of kernels with different shared-memory carveouts cannot share an
-        // SM: the concurrent kernel (the tensor-core contraction) needs ~200 KB
-        CU_TRY(drv.FuncSetAttribute(k->fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100));
-        k->carveout_max = true;
-    }
+    long long cap = (long long)k->blocks_per_sm * c->num_sms;
     int grid = (int)std::max(1ll, std::min(want, cap));
     void *args[] = {&P};
     if (k->pdl && c->pipelined) {
@@ -543,11 +529,6 @@ up_status up_ctx_destroy(up_ctx *c) {
     for (auto &kv : c->pow10_dev) cudaFree(kv.second);
     cudaFree(c->d_ws);
     cudaFree(c->d_ticket);
-    if (c->d_ws2) cudaFree(c->d_ws2);
-    if (c->d_ticket2) cudaFree(c->d_ticket2);
-    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
-    if (c->ev_join) cudaEventDestroy(c->ev_join);
-    if (c->side) cudaStreamDestroy(c->side);
     cudaFree(c->d_flags);
     if (c->d_stage) cudaFree(c->d_stage);
     if (c->d_scratch) cudaFree(c->d_scratch);
@@ -952,11 +933,7 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             const int T = (int)pl.prods.size() + (pl.rest_kernel ? 1 : 0);
             const size_t need = (size_t)T * (size_t)LAs;
             if (need > c->parts_words) {
-                if (c->d_parts) {
-                    CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream));
-                    if (c->side) CUDA_TRY(cudaStreamSynchronize(c->side));
-                    CUDA_TRY(cudaFree(c->d_parts));
-                }
+                if (c->d_parts) { CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream)); CUDA_TRY(cudaFree(c->d_parts)); }
                 CUDA_TRY(cudaMalloc(&c->d_parts, sizeof(uint32_t) * need * 2));
                 c->parts_words = need * 2;
             }
@@ -965,40 +942,14 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             P.ws = c->d_ws;
             P.ticket = c->d_ticket;
             P.flags = c->d_flags;
-            // quad columns: the tensor-core contraction (a few warps and the
-            // shared-memory stages, HBM-bound) runs on the side stream while the
-            // integer-bound rest kernel fills the SMs' remaining block slots on
-            // the caller's stream; joined before the combine (UP_SERIAL_SPLIT:
-            // one stream, back to back)
-            bool overlap = pl.rest_kernel != nullptr && !getenv("UP_SERIAL_SPLIT");
-            for (size_t q = 0; q < pl.prods.size() && overlap; ++q)
-                overlap = !pl.cc_kernels[q] && cols[pl.prods[q].col_a].layout == UP_LAYOUT_QUADS;
-            cudaStream_t tcs = (cudaStream_t)stream;
-            unsigned long long *tws = c->d_ws;
-            uint32_t *ttk = c->d_ticket;
-            if (overlap) {
-                if (!c->side) {
-                    CUDA_TRY(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
-                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
-                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
-                    CUDA_TRY(cudaMalloc(&c->d_ws2, sizeof(unsigned long long) * 2 * 1024));
-                    CUDA_TRY(cudaMemset(c->d_ws2, 0, sizeof(unsigned long long) * 2 * 1024));
-                    CUDA_TRY(cudaMalloc(&c->d_ticket2, 64));
-                    CUDA_TRY(cudaMemset(c->d_ticket2, 0, 64));
-                    CUDA_TRY(cudaDeviceSynchronize());
-                }
-                CUDA_TRY(cudaEventRecord(c->ev_fork, (cudaStream_t)stream));
-                CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_fork, 0));
-                tcs = c->side; tws = c->d_ws2; ttk = c->d_ticket2;
-            }
             int ti = 0;
             for (size_t q = 0; q < pl.prods.size(); ++q) {
                 const SplitTerm &st = pl.prods[q];
                 const up_column &ca = cols[st.col_a], &cb = cols[st.col_b];
                 if (!pl.cc_kernels[q]) {
                     auto tc = ca.layout == UP_LAYOUT_QUADS ? upk_launch_contract_tq : upk_launch_contract_tc;
-                    CUDA_TRY(tc(ca.data, ca.ld, ca.limbs, cb.data, cb.ld, cb.limbs, cols[0].n, st.sign, tws, ttk,
-                                c->d_parts + (size_t)ti++ * LAs, LAs, c->num_sms, tcs));
+                    CUDA_TRY(tc(ca.data, ca.ld, ca.limbs, cb.data, cb.ld, cb.limbs, cols[0].n, st.sign, c->d_ws, c->d_ticket,
+                                c->d_parts + (size_t)ti++ * LAs, LAs, c->num_sms, (cudaStream_t)stream));
                     c->launches++;
                     continue;
                 }
@@ -1007,12 +958,7 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             }
             if (pl.rest_kernel) {
                 P.result = c->d_parts + (size_t)ti++ * LAs;
-                // one block slot per SM left to the contraction CTA
-                if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream, overlap ? 1 : 0)) return s;
-            }
-            if (overlap) {
-                CUDA_TRY(cudaEventRecord(c->ev_join, c->side));
-                CUDA_TRY(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_join, 0));
+                if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream)) return s;
             }
             if (pl.rest_kernel && pl.rest_scale > 0) {
                 const uint32_t *d_sc = nullptr;

@@ -114,15 +114,11 @@ def test_quad_contraction_empty():
 CFG3 = [(200, 50), (500, 75), (1000, 100)]
 
 
-@pytest.mark.parametrize("serial", [False, True], ids=["overlap", "serial"])
 @pytest.mark.parametrize("ps", CFG3, ids=lambda t: f"p{t[0]}")
 @pytest.mark.parametrize("n", [1, 1000, 4099])
-def test_cfg3_sum_quads(ps, n, serial, monkeypatch):
-    """cfg3's SUM(c1*c2 - c3/c4) over quad columns (tensor-core contraction on
-    the side stream concurrently with the fused top-limb division, or both on
-    one stream with UP_SERIAL_SPLIT) == the oracle"""
-    if serial:
-        monkeypatch.setenv("UP_SERIAL_SPLIT", "1")
+def test_cfg3_sum_quads(ps, n):
+    """cfg3's SUM(c1*c2 - c3/c4) over quad columns (tensor-core contraction +
+    the fused top-limb division reading quads) == the oracle"""
     types = [ps] * 4
     host = G.gen_cols(n, types, config=3, nonzero_lead_cols=(3,))
     want, P, S = oracle.eval_sum("c1*c2 - c3/c4", G.to_oracle(host, types), n=n, threads=8)
@@ -135,8 +131,9 @@ def test_cfg3_sum_quads(ps, n, serial, monkeypatch):
 
 def test_cfg3_quads_back_to_back_pipelined():
     """K split SUMs back to back on one stream with pipelined (PDL) launches:
-    the side-stream contraction and the rest kernel of consecutive steps share
-    the partials buffer and the workspaces -- every result must be the oracle's"""
+    the contraction, the rest kernel and the combine of consecutive steps
+    share the partials buffer and the workspace -- every result must be the
+    oracle's"""
     import torch
     types = [(200, 50)] * 4
     n = 70001

@@ -3,8 +3,10 @@
 cfg3 (DECIMAL(200,50) x 4, 12.5M rows): the tensor-core contraction
 SUM(c1*c2) alone, the rest SUM(c3/c4) alone, the two back to back on one
 stream, the two on two streams from two contexts (separate workspaces), and
-the library's split step (side stream inside up_sum_expr).  Prints one JSON
-line.  Measurement tool only (no product code path).
+the library's split step.  Prints one JSON line.  Measurement tool only (no
+product code path).  Round-2 result (profiles/r02_s28, r02_s31): two streams
+0.69-0.90 ms vs 0.80-0.86 back to back, varying from run to run with the
+block placement -- the library keeps the kernels on one stream.
 
     python tools/probe_overlap.py [--rows N] [--reps K]
 """
@@ -73,8 +75,6 @@ def main():
 
     r = {"p": a.p, "rows": n, "rest_layout": a.rest_layout, "tc_ms": t(tc), "rest_ms": t(rest), "serial_ms": t(both_serial),
          "two_streams_ms": t(both_streams), "split_step_ms": t(split)}
-    os.environ["UP_SERIAL_SPLIT"] = "1"
-    r["split_serial_ms"] = t(split)
     print(json.dumps(r))
 
 
