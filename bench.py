@@ -252,9 +252,15 @@ class ExprWorkload(Workload):
         tc_row = _col_bytes(p, self.args.layout)
         tc_bytes = 2 * tc_row * self.rows
         ach = tc_bytes / (t_tc / 1e3) / 1e9
-        mag = lambda k: max(1, (10 ** k).bit_length() // 32 + 1)   # noqa: E731
-        nu = mag(p + s + 4)
-        div_products = L * mag(s + 4) + (nu - L + 1) * L
+        # the rest kernel's arithmetic: the top-limb decision per row (DESIGN §5,
+        # up_dev.cuh div_top_decide): ah x C (T x NC limb products) and NQ quotient
+        # limbs of T products each (3-by-2 step + multiply-subtract); NC = limbs of
+        # C = 10^(s+4), NQ = limbs of the quotient type, T = max(NC, NQ) + 1 -- the
+        # products the kernel performs, not the SURVEY's full-division count
+        nc = ((10 ** (s + 4)).bit_length() + 31) // 32
+        nq = up.limbs(max(s + 5, 1))
+        T = max(nc, nq) + 1
+        div_products = T * (nc + nq)
         pk, src = _product_peak()
         rest_ach = div_products * self.rows / (t_rest / 1e3)
         return {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
@@ -267,8 +273,8 @@ class ExprWorkload(Workload):
                      "alg_bytes": tc_bytes, "achieved_gbs": round(ach, 1), "frac": round(ach / peak, 4)},
                     {"kernel": "upk rest (SUM(-c3/c4), top-limb division)", "ms": round(t_rest, 5), "bound": "alu",
                      "alg_products": div_products * self.rows,
-                     "alg_unit": f"{div_products} limb products/row (SURVEY 8d division count; the kernel decides "
-                                 "most quotients from the top limbs and does fewer)",
+                     "alg_unit": f"{div_products} limb products/row (top-limb decision: T={T} limbs x (C {nc} + "
+                                 f"quotient {nq} limbs))",
                      "achieved_T_products_s": round(rest_ach / 1e12, 4), "frac": round(rest_ach / pk, 4),
                      "peak_source": src}],
                 "step_ms": round(step_ms, 5),
