@@ -104,7 +104,8 @@ typedef struct {
  *     box of this layout lands in shared memory as the tensor cores' MN-major
  *     core matrices (16 digit bytes x 8 rows) with the sign digit included,
  *     so SUM(c_a*c_b) feeds tcgen05 straight from the copies (SURVEY §8a rows
- *     a6/a11; contract_tc.cu).  Read by up_eval_expr / up_sum_expr / up_sum /
+ *     a6/a11; contract_tc.cu; calls below 2^30 rows -- beyond, the product
+ *     stays in the fused per-row kernel).  Read by up_eval_expr / up_sum_expr / up_sum /
  *     up_filter (every generated kernel reads quads with 16-byte loads);
  *     ingestion and read-back convert through limb planes in the ctx scratch.
  *     Other entry points return UP_E_UNSUPPORTED for quad inputs.

@@ -740,6 +740,7 @@ cudaError_t upk_launch_contract_tc(const uint32_t *A, long long lda, int La, con
 cudaError_t upk_launch_contract_tq(const uint32_t *A, long long lda, int La, const uint32_t *B, long long ldb, int Lb,
                                    long long n, int sign, unsigned long long *ws, uint32_t *ticket, uint32_t *result,
                                    int LA, int num_sms, cudaStream_t st) {
+    if (n >= (1ll << 30)) return cudaErrorInvalidValue;   // TMA coordinate 2 * row must fit int32
     TqArgs P;
     P.n = n; P.La = La; P.Lb = Lb;
     P.Ga = (La + 1 + 3) / 4; P.Gb = (Lb + 1 + 3) / 4;

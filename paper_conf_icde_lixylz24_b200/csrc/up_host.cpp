@@ -882,7 +882,10 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
     if (try_split && !getenv("UP_NO_SPLIT")) {
         // the split plan (terms, kernels) is cached per (expression, column types, N, knobs):
         // typing, optimising and splitting cost host time on every call otherwise
-        std::string pkey = key_of("splitplan", expr, cols, ncols, 0) + "|" + std::to_string(N) + (use_tc ? "|tc" : "");
+        // quad contractions address rows as 2 u64 per row in 32-bit TMA coordinates
+        const bool quad_tc = use_tc && cols[0].n < (1ll << 30);
+        std::string pkey = key_of("splitplan", expr, cols, ncols, 0) + "|" + std::to_string(N) + (use_tc ? "|tc" : "") +
+                           (quad_tc ? "|qtc" : "");
         auto pit = c->plans.find(pkey);
         if (pit == c->plans.end()) {
             SplitPlan pl;
@@ -902,7 +905,7 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
                     const bool tc_ok = use_tc && upk_contract_tc_slots(La, Lb) <= kWsSlots;
                     // quad columns: the tensor-core contraction reads both operands as quads;
                     // otherwise the whole SUM stays in the fused kernel
-                    if ((qa || qb) && !(qa && qb && tc_ok)) { pl.split = false; break; }
+                    if ((qa || qb) && !(qa && qb && tc_ok && quad_tc)) { pl.split = false; break; }
                     if (!tc_ok) {
                         std::string key = "contract|" + std::to_string(La) + "|" + std::to_string(Lb) + "|" + std::to_string(LAs) +
                                           "|" + std::to_string(st.sign) + "|" + std::to_string(st.col_a) + "|" + std::to_string(st.col_b);
