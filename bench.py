@@ -147,6 +147,23 @@ class Workload:
         self.e2e_rows = min(rows, E2E_MAX_ROWS)
 
 
+def _h2d_copy_gbs(nbytes, reps=5):
+    """pinned host -> device copy bandwidth for nbytes (the e2e path's link)"""
+    import torch
+    nbytes = max(1 << 20, min(int(nbytes), 1 << 30))
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    d.copy_(h, non_blocking=True)
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(reps):
+        d.copy_(h, non_blocking=True)
+    b.record()
+    torch.cuda.synchronize()
+    return round(nbytes * reps / (a.elapsed_time(b) / 1e3) / 1e9, 2)
+
+
 def _col_bytes(p, layout):
     from paper_conf_icde_lixylz24_b200 import up
     return {"compact": up.compact_bytes(p), "quads": 16 * up.quads(p)}.get(layout, 4 * up.limbs(p))
@@ -750,7 +767,10 @@ def main():
         assert up.format_decimal(res_host.tolist(), wl.S) == result, "e2e result differs from the resident run"
     h2d = sum(hb.numel() for hb in host)
     e2e = {"value": e2e_global / (ems / K2 / 1e3), "unit": "tuples/s", "h2d_bytes_per_step": h2d,
-           "d2h_bytes_per_step": LA * 4, "ms_per_step": ems / K2}
+           "d2h_bytes_per_step": LA * 4, "ms_per_step": ems / K2,
+           # the host link is the e2e roofline: the rows' bytes over the step time,
+           # beside a plain pinned host->device copy of the same size measured here
+           "h2d_gbs": round(h2d / (ems / K2 / 1e3) / 1e9, 2), "h2d_copy_gbs": _h2d_copy_gbs(h2d)}
     if wl.e2e_rows < rows:
         e2e["rows"] = f"first {wl.e2e_rows} rows of each rank's shard ({e2e_global} in total)"
 

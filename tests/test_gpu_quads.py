@@ -214,3 +214,21 @@ def test_quads_refused_where_unsupported():
         c.eval_tpi("+", x, x, tpi=4)
     with pytest.raises(up.UpError):
         c.group_aggregate([("SUM", "c1")], [x])
+
+
+@pytest.mark.parametrize("op", ["<", "=", ">="])
+@pytest.mark.parametrize("lhs,rhs,types,n", [
+    ("c1", "c2", [(4, 1), (3, 2)], 1001),                        # narrow: 4 rows per thread
+    ("c1 / c2", "c3", [(200, 50), (200, 50), (6, 4)], 503),       # top-limb division over quads
+    ("c1 * c2 - c3", "0", [(60, 10), (50, 20), (100, 30)], 301),
+])
+def test_quads_filter_parity(op, lhs, rhs, types, n):
+    """WHERE over quad columns (up_filter reads quads like planes) == the oracle"""
+    import torch
+    host = G.gen_cols(n, types, config=11, nonzero_lead_cols=(1,) if "/" in lhs else ())
+    c = G.ctx()
+    g = [c.column_from_host_bin(p, s, m, ng, layout="quads") for (m, ng), (p, s) in zip(host, types)]
+    pre = np.where(np.arange(n) % 11 == 0, -1, 0).astype(np.int32)
+    ids = c.filter(lhs, op, rhs, g, torch.as_tensor(pre, device="cuda"))
+    c.check()
+    assert ids.cpu().tolist() == oracle.filter_ids(lhs, op, rhs, G.to_oracle(host, types), pre.tolist())
