@@ -127,6 +127,8 @@ up_status fail(up_status st, const char *fmt, ...) {
 
 constexpr int kThreads = 256;
 constexpr int kWsSlots = 1 << 16;
+constexpr int kIngestChunks = 8;          // host ingestion: copy / convert pipeline depth
+constexpr size_t kIngestChunkMin = 16u << 20;   // bytes per chunk at least
 constexpr int kContractMinProducts = 100;   // row contraction only for compute-bound products
 constexpr long kSplitAutoProducts = 80 * 80;  // automatic split from this product size on
 constexpr int kWideMinLimbs = 257;  // warp-per-row only beyond this (per-thread measured faster at p <= 1000)
@@ -176,6 +178,10 @@ struct up_ctx {
     uint64_t launches = 0;
     double jit_ms = 0.0;
     bool pipelined = false;   // up_set_pipelined: PDL launches of the fused SUM kernels
+    // host ingestion: a copy stream and per-chunk events, so the H2D copy of
+    // chunk k+1 overlaps the conversion / range check of chunk k
+    cudaStream_t copy_st = nullptr;
+    cudaEvent_t chunk_ev[kIngestChunks] = {};
     std::mutex mu;
 };
 
@@ -531,6 +537,8 @@ up_status up_ctx_destroy(up_ctx *c) {
     cudaFree(c->d_ticket);
     cudaFree(c->d_flags);
     if (c->d_stage) cudaFree(c->d_stage);
+    for (cudaEvent_t e : c->chunk_ev) if (e) cudaEventDestroy(e);
+    if (c->copy_st) cudaStreamDestroy(c->copy_st);
     if (c->d_scratch) cudaFree(c->d_scratch);
     if (c->d_parts) cudaFree(c->d_parts);
     delete c;
@@ -669,24 +677,62 @@ up_status up_column_from_device_compact(up_ctx *c, const uint8_t *d_bytes, up_co
     return UP_OK;
 }
 
+// Host compact rows -> dst in chunks of rows: the copy of chunk k+1 (ctx copy
+// stream) overlaps the conversion or range check of chunk k (the caller's
+// stream, after the chunk's event), so only the last chunk's kernel is
+// exposed behind the host link.
 up_status up_column_from_host_compact(up_ctx *c, const uint8_t *bytes, up_column *dst, void *stream) {
     if (!c || !bytes) return fail(UP_E_INVAL, "null argument");
     if (up_status s = check_column(dst, "dst")) return s;
     if (dst->n == 0) return UP_OK;
     cudaStream_t st = (cudaStream_t)stream;
-    const size_t nb = (size_t)up_compact_bytes(dst->p) * (size_t)dst->n;
-    if (dst->layout == UP_LAYOUT_COMPACT) {   // rows land in place: H2D + range check, no conversion
-        CUDA_TRY(cudaMemcpyAsync(dst->data, bytes, nb, cudaMemcpyHostToDevice, st));
-        if (up_status s = up_column_from_device_compact(c, (const uint8_t *)dst->data, dst, stream)) return s;
-        CUDA_TRY(cudaStreamSynchronize(st));   // up.h: host buffer reusable on return
-        return UP_OK;
+    const int Lb = up_compact_bytes(dst->p);
+    const long long n = dst->n;
+    const size_t nb = (size_t)Lb * (size_t)n;
+    std::lock_guard<std::mutex> g(c->mu);
+    if (!c->copy_st) {
+        CUDA_TRY(cudaStreamCreateWithFlags(&c->copy_st, cudaStreamNonBlocking));
+        for (cudaEvent_t &e : c->chunk_ev) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     }
-    {
-        std::lock_guard<std::mutex> g(c->mu);
+    const uint32_t *bound = nullptr;
+    if (up_status s = pow10_device(c, dst->p, &bound)) return s;
+    // destination of the raw rows: in place (compact column) or the ctx stage
+    uint8_t *raw = nullptr;
+    if (dst->layout == UP_LAYOUT_COMPACT) raw = (uint8_t *)dst->data;
+    else {
         if (up_status s = ensure_stage(c, nb, st)) return s;
-        CUDA_TRY(cudaMemcpyAsync(c->d_stage, bytes, nb, cudaMemcpyHostToDevice, st));
+        raw = (uint8_t *)c->d_stage;
     }
-    if (up_status s = up_column_from_device_compact(c, (const uint8_t *)c->d_stage, dst, stream)) return s;
+    uint32_t *planes = dst->data;
+    long long ld = dst->ld;
+    if (dst->layout == UP_LAYOUT_QUADS) {   // via limb planes in the ctx scratch
+        ld = (n + 3) & ~3ll;
+        if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)dst->limbs * (size_t)ld, (void **)&planes)) return s;
+    }
+    const int nck = (int)std::max<size_t>(1, std::min<size_t>(kIngestChunks, nb / kIngestChunkMin));
+    // the copy stream starts after the caller's prior work (the stage may still be read)
+    CUDA_TRY(cudaEventRecord(c->chunk_ev[0], st));
+    CUDA_TRY(cudaStreamWaitEvent(c->copy_st, c->chunk_ev[0], 0));
+    for (int k = 0; k < nck; ++k) {
+        // chunk boundaries on 256-row multiples: 4-byte-aligned compact rows for the kernel's word loads
+        const long long r0 = (n * k / nck) & ~255ll, r1 = k + 1 == nck ? n : (n * (k + 1) / nck) & ~255ll;
+        if (r1 == r0) continue;
+        CUDA_TRY(cudaMemcpyAsync(raw + (size_t)r0 * Lb, bytes + (size_t)r0 * Lb, (size_t)(r1 - r0) * Lb,
+                                 cudaMemcpyHostToDevice, c->copy_st));
+        CUDA_TRY(cudaEventRecord(c->chunk_ev[k], c->copy_st));
+        CUDA_TRY(cudaStreamWaitEvent(st, c->chunk_ev[k], 0));
+        if (dst->layout == UP_LAYOUT_COMPACT) {   // rows landed in place: range check only
+            CUDA_TRY(upk_launch_from_compact(raw + (size_t)r0 * Lb, Lb, r1 - r0, bound, dst->limbs, nullptr, 0, c->d_flags, st));
+        } else {
+            CUDA_TRY(upk_launch_from_compact(raw + (size_t)r0 * Lb, Lb, r1 - r0, bound, dst->limbs, planes + r0, ld,
+                                             c->d_flags, st));
+            if (dst->layout == UP_LAYOUT_QUADS) {
+                CUDA_TRY(upk_launch_planes_to_quads(planes + r0, dst->limbs, ld, r1 - r0, dst->data + 4 * r0, dst->ld, st));
+                c->launches++;
+            }
+        }
+        c->launches++;
+    }
     CUDA_TRY(cudaStreamSynchronize(st));   // up.h: host buffer reusable on return
     return UP_OK;
 }

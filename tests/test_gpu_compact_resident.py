@@ -112,3 +112,35 @@ def test_compact_unsupported_entry_points():
     with pytest.raises(up.UpError) as ei:
         c.sin_taylor(x, 20)
     assert ei.value.name == "UNSUPPORTED"
+
+
+@pytest.mark.parametrize("layout", ["planes", "quads", "compact"])
+def test_chunked_host_compact_ingestion(layout):
+    """up_column_from_host_compact pipelines large inputs in chunks (the copy of
+    chunk k+1 beside the conversion of chunk k, 256-row chunk boundaries): a
+    9M-row column (8 chunks) must equal the one-kernel device ingestion byte
+    for byte, and a range error in a middle chunk must still raise RANGE."""
+    import torch
+    from gen import device as gdev
+    from paper_conf_icde_lixylz24_b200 import up
+    c = G.ctx()
+    n, p, s = 9_000_003, 35, 5
+    mag, neg = gdev.uniform_decimal(n, p, 2, 1)
+    ref = c.column_from_device_bin(p, s, mag, neg)
+    del mag, neg
+    rows = c.column_to_compact(ref)
+    col = c.column_from_compact(p, s, torch.from_numpy(rows).pin_memory(), n=n, layout=layout)
+    c.check()
+    assert np.array_equal(c.column_to_compact(col), rows)
+    got, _, _ = G.gpu_sum_string("c1", [col])
+    want, _, _ = G.gpu_sum_string("c1", [ref])
+    assert got == want
+    Lb = up.compact_bytes(p)
+    bad = rows.copy()
+    r = 4_500_001                                   # inside the 5th of 8 chunks
+    bad[r * Lb:(r + 1) * Lb] = 0xFF
+    bad[(r + 1) * Lb - 1] = 0x7F                    # magnitude 2^119 - 1 >= 10^35, positive
+    c.column_from_compact(p, s, torch.from_numpy(bad).pin_memory(), n=n, layout=layout)
+    with pytest.raises(up.UpError) as ei:
+        c.check()
+    assert ei.value.name == "RANGE"
