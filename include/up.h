@@ -152,7 +152,10 @@ up_status up_column_to_host_bin(up_ctx *ctx, const up_column *col, uint32_t *mag
  * magnitude little-endian in the low 8*Lb-1 bits and the sign in the top bit
  * of the last byte (-1.23 in DECIMAL(10,2) = {123,0,0,0,0x80}).  Rows are
  * contiguous (row i at bytes[i*Lb]).  _host_: host buffer staged through the
- * ctx (same lifetime rule as _host_bin); _device_: device buffer;
+ * ctx (same lifetime rule as _host_bin; inputs of >= 32 MB are copied in up to
+ * 8 chunks on a ctx-owned copy stream, each chunk converted / range-checked on
+ * `stream` as soon as it lands -- pinned memory makes the copies asynchronous);
+ * _device_: device buffer;
  * to_host_compact synchronises the stream.  Range errors set RANGE.
  */
 int32_t up_compact_bytes(int32_t p);
