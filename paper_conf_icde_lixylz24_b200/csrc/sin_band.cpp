@@ -44,25 +44,6 @@ namespace uph {
 
 namespace {
 
-// bank-conflict-minimising padded row stride (words) for one access
-// instruction of the warp: lane (g, b) touches word (base - D b) of row slot g
-// (D = digit distance between consecutive band lanes); elt = 1 (u32) or 2 (u64)
-int pick_stride(int R, int G, int D, int elt) {
-    int best = R, bestc = 1 << 30;
-    for (int rs = R; rs < R + 64; ++rs) {
-        int cnt[32] = {0};
-        for (int b = 0; b < G; ++b)
-            for (int g = 0; g < 32 / G; ++g) {
-                const long long idx = (long long)(1000 - D * b) * rs + g;
-                for (int e = 0; e < elt; ++e) cnt[(idx * elt + e) & 31]++;
-            }
-        int mx = 0;
-        for (int i = 0; i < 32; ++i) mx = std::max(mx, cnt[i]);
-        if (mx < bestc) { bestc = mx; best = rs; }
-    }
-    return best;
-}
-
 std::string hex_arr(const std::vector<uint32_t> &w) {
     std::ostringstream o;
     o << "{";
@@ -360,11 +341,12 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
         kmax += 2;
     }
     int G = G_req;
-    // lanes per row (measured, profiles/r02_s16, 100k rows): P = 2000 (W = 212) G = 4
-    // 5.7e6 rows/s (G = 8: 4.8e6), P = 3000 / 5000 G = 8 (2.5e6 / 9.9e5; G = 16: 2.3e6 /
-    // 9.3e5), P = 10000 G = 32 (3.1e5; G = 16: 2.3e5), P = 20000 G = 32.  Fewer lanes: less
-    // pipeline fill (DELTA (G - 1) steps per band); more: more rows resident (shared memory)
-    if (G <= 0) G = W <= 250 ? 4 : W <= 700 ? 8 : 32;
+    // lanes per row (measured with packed row slots, profiles/r02_s40): P = 2000 (W = 213)
+    // G = 4 5.87e6 rows/s (G = 8: 5.19e6), P = 3000 G = 4 2.78e6 (G = 8: 2.50e6), P = 5000
+    // G = 8 1.23e6 (G = 4: 0.89e6, G = 16: 1.12e6), P = 10000 G = 16 3.41e5 (G = 32:
+    // 3.10e5), P = 20000 G = 32 9.53e4 (G = 16: 7.36e4).  Fewer lanes: less pipeline
+    // fill (DELTA (G - 1) steps per band); more: more rows resident (shared memory)
+    if (G <= 0) G = W <= 350 ? 4 : W <= 700 ? 8 : W <= 1500 ? 16 : 32;
     if (G != 1 && G != 2 && G != 4 && G != 8 && G != 16 && G != 32) { err = "band sine: G must divide 32"; return ""; }
     // one row per lane group (two rows per lane were measured slower, profiles/r02_s5)
     const int R = 32 / G;
@@ -398,7 +380,10 @@ std::string gen_sin_kernel_band(int P, int p, int s, int Lout, int LA, bool sum,
     if (!split) NR = (int)std::max(1.0, std::floor(std::pow(2.0, 61.0 - per_row)));
     else NR = (int)std::max(1.0, std::floor(std::pow(2.0, 61.0 - (std::log2((double)kmax + G) + 33))));
     // lanes of one step touch digits 2 DELTA apart (lane b) in rows g
-    const int RSY = pick_stride(R, G, 2 * DELTA, 1), RSS = pick_stride(R, G, 2 * DELTA, 2);
+    // row slots packed (stride R): padding the strides against the 2-way bank
+    // conflicts of lanes b and b + 4 cost more resident rows than it saved
+    // (P = 5000: 0.99e6 -> 1.23e6 rows/s without it, P = 2000 +1 %, r02_s39)
+    const int RSY = R, RSS = R;
     // negative (even-k) terms have o_k = c for every even k (s = 8: o = 16; s = 0: o = 0)
     bool negsh0 = true;
     for (int kk = 2; kk <= 64; kk += 2) negsh0 = negsh0 && (((2 * s * (kk - 1)) & 31) == csc);
