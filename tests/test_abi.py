@@ -124,3 +124,29 @@ def test_tpi_kernels_compile_for_sm100a():
     for alg in ("long", "newton"):
         for types in ([(40, 5), (30, 2)], [(200, 50), (200, 50)], [(20, 0), (9, 0)]):
             up.nvrtc_compile(up.gen_tpi_source("/", types, 1, alg))
+
+
+@pytest.mark.parametrize("variant,expr,types,layouts", [
+    ("sum", "c1+c2", [(17, 5), (14, 2)], ["quads", "quads"]),                  # 4 rows per thread, 16-byte quad loads
+    ("sum", "c1/c2", [(200, 50)] * 2, ["quads", "quads"]),                     # top-limb window from quads, out-of-line fallback
+    ("eval", "c1*c2 - c3/c4", [(200, 50)] * 4, ["quads", "planes", "compact", "quads"]),
+])
+def test_quad_layout_kernels_compile_for_sm100a(variant, expr, types, layouts, tmp_path):
+    """limb-quad columns (up.h UP_LAYOUT_QUADS): the generated kernels read
+    them with 16-byte loads and compile for sm_100a; the division's decision
+    window loads whole quads and its full-division fallback is out of line"""
+    src = up.gen_source(variant, expr, types, 1_000_000, layouts=layouts)
+    assert "ld_quads<" in src or "reinterpret_cast<const uint4 *>(g" in src
+    if expr == "c1/c2":   # both division operands are columns read lazily: fallback out of line
+        assert "__noinline__" in src and "div_top_decide<" in src
+    log = up.nvrtc_compile(src, str(tmp_path / "q.cubin"))
+    assert (tmp_path / "q.cubin").stat().st_size > 0, log
+    if expr == "c1+c2":
+        regs, spills = _regs(log)
+        assert spills == 0 and regs <= 64, log
+
+
+def test_quads_abi():
+    """up_quads(p) = ceil((up_limbs(p) + 1) / 4): the sign-flag limb included"""
+    for p in (1, 9, 18, 38, 76, 153, 200, 307, 1000):
+        assert up.quads(p) == (up.limbs(p) + 1 + 3) // 4
