@@ -42,6 +42,15 @@ def _worker(rank, world, port, kind, n, q):
             mag, neg = gdev.uniform_decimal(hi - lo, p, 2, k + 1, row0=lo)
             cols.append(ctx.column_from_device_bin(p, s, mag, neg))
         ss = ShardedSum.expr(ctx, "c1+c2", cols, n)
+    elif kind == "cfg3q":
+        # cfg3's SUM(c1*c2 - c3/c4) over limb quads: every rank runs the split
+        # (tensor-core contraction + top-limb division) on its shard
+        types = [(200, 50)] * 4
+        cols = []
+        for k, (p, s) in enumerate(types):
+            mag, neg = gdev.uniform_decimal(hi - lo, p, 3, k + 1, row0=lo, nonzero_lead=(k == 3))
+            cols.append(ctx.column_from_device_bin(p, s, mag, neg, layout="quads"))
+        ss = ShardedSum.expr(ctx, "c1*c2 - c3/c4", cols, n)
     elif kind == "modexp":
         N, _, _ = synth.rsa_modulus(256)
         mag, neg = gdev.uniform_range(synth.SEED, synth.stream_id(4, 0), hi - lo, 0, N - 1, signed=False, row0=lo)
@@ -105,6 +114,11 @@ def _oracle_whole(kind, n):
         host = [synth.uniform_decimal(n, p, 2, k + 1) for k, (p, s) in enumerate(types)]
         return oracle.eval_sum("c1+c2", [oracle.Column(p, s, m, g) for (m, g), (p, s) in zip(host, types)],
                                threads=4)[0]
+    if kind == "cfg3q":
+        types = [(200, 50)] * 4
+        host = [synth.uniform_decimal(n, p, 3, k + 1, nonzero_lead=(k == 3)) for k, (p, s) in enumerate(types)]
+        return oracle.eval_sum("c1*c2 - c3/c4", [oracle.Column(p, s, m, g) for (m, g), (p, s) in zip(host, types)],
+                               threads=4)[0]
     if kind == "modexp":
         N, _, _ = synth.rsa_modulus(256)
         m, g = synth.rsa_messages(n, N)
@@ -115,7 +129,7 @@ def _oracle_whole(kind, n):
 
 @pytest.mark.parametrize("kind,n,world", [("expr", 1, 2), ("expr", 100_003, 2), ("modexp", 3001, 2),
                                           ("sin", 2049, 2), ("expr", 50_000, 3), ("group", 30_001, 2),
-                                          ("group", 7, 3)])
+                                          ("group", 7, 3), ("cfg3q", 4001, 2)])
 def test_sharded_sum_two_processes_one_gpu(kind, n, world):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
