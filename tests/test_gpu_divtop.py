@@ -54,7 +54,9 @@ def _rows(p1, s1, p2, s2, n_random, seed):
 
 
 @pytest.mark.parametrize("t1,t2", [((200, 50), (200, 50)), ((500, 75), (500, 75)), ((1000, 100), (1000, 100)),
-                                   ((300, 0), (250, 10)), ((250, 20), (200, 60))])
+                                   ((300, 0), (250, 10)), ((250, 20), (200, 60)),
+                                   # small decision windows: T = 2 (C and q one limb each), T = 3
+                                   ((20, 0), (20, 2)), ((40, 3), (38, 1)), ((30, 5), (30, 5))])
 def test_divtop_rows_and_sum(t1, t2):
     (p1, s1), (p2, s2) = t1, t2
     A, B = _rows(p1, s1, p2, s2, 300, seed=p1 * 7 + p2)
