@@ -202,6 +202,9 @@ def test_quads_compact_ingest_and_readback():
     assert c.column_to_ints(q) == vals
     assert bytes(c.column_to_compact(q)) == bytes(comp)
     assert q.layout == up.LAYOUT_QUADS
+    import torch   # the device-buffer entry point (up_column_from_device_compact) into quads
+    qd = c.column_from_compact(p, 0, torch.from_numpy(comp).cuda(), n=n, layout="quads")
+    assert c.column_to_ints(qd) == vals
 
 
 def test_quads_refused_where_unsupported():
