@@ -36,6 +36,30 @@ def _dev_cols(n, types, config, lead=()):
     return cols
 
 
+@pytest.mark.parametrize("name", ["cfg3_p200", "cfg3_p500", "cfg3_p1000"])
+def test_full_size_cfg3_quads_vs_golden(name):
+    """cfg3 as the bench runs it -- limb-quad columns, the tensor-core
+    contraction fed straight from TMA (148 CTAs, several accumulation windows
+    each) plus the top-limb division -- against the oracle's full SUM"""
+    import torch
+    g = _gold(name)
+    w = g["workload"]
+    types = [tuple(t) for t in w["types"]]
+    lead = tuple(w.get("lead", ()))
+    c = G.ctx()
+    cols = []
+    for k, (p, s) in enumerate(types):
+        mag, neg = gdev.uniform_decimal(w["rows"], p, w["config"], k + 1, nonzero_lead=(k in lead))
+        cols.append(c.column_from_device_bin(p, s, mag, neg, layout="quads"))
+        del mag, neg
+    c.check()
+    got, P, S = G.gpu_sum_string(w["expr"], cols)
+    assert (P, S) == (g["p"], g["s"])
+    assert got == g["sum"]
+    del cols
+    torch.cuda.empty_cache()
+
+
 def _gold(name):
     if name not in GOLD:   # oracle runs of ~0.5 h each are written off the GPU box (tools/make_golden.py)
         pytest.skip(f"golden entry {name} not computed yet: run tools/make_golden.py --only {name}")
