@@ -358,8 +358,30 @@ class ModexpWorkload(ExprWorkload):
     def kernel(self, out):
         self.ctx.modexp_sum(self.cols[0], self.e, self.N, self.n_global, out=out)
 
+    # e2e streamed in row chunks (the public API composed): the ingestion of
+    # chunk k+1 (its H2D copy on the ctx copy stream) runs while the modexp SUM
+    # of chunk k computes; the chunk partials (typed with the global N) are
+    # added by up_sum_combine.  The host link and the integer pipes overlap.
+    E2E_CHUNKS = 8
+
+    def e2e_ingest(self, host):
+        self._e2e_host = host
+
     def e2e_kernel(self, out):
-        self.ctx.modexp_sum(self.e2e_cols[0], self.e, self.N, self.n_global, out=out)
+        import torch
+        from paper_conf_icde_lixylz24_b200 import up
+        hb, col = self._e2e_host[0], self.e2e_cols[0]
+        Lb = up.compact_bytes(self.d)
+        n, C = col.n, self.E2E_CHUNKS
+        if getattr(self, "_parts", None) is None:
+            self._parts = torch.empty((C, self.LA), dtype=torch.int32, device="cuda")
+        for k in range(C):
+            r0 = (n * k // C) & ~255
+            r1 = n if k == C - 1 else (n * (k + 1) // C) & ~255
+            view = col.rows(r0, r1)
+            self.ctx.column_from_compact(self.d, 0, hb[r0 * Lb:r1 * Lb], n=r1 - r0, out=view)
+            self.ctx.modexp_sum(view, self.e, self.N, self.n_global, out=self._parts[k])
+        self.ctx.sum_combine(self._parts, self.LA, out=out)
 
     def roofline(self, kernel_ms, peaks):
         n = (self.N.bit_length() + 31) // 32

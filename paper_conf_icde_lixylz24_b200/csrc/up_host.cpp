@@ -710,9 +710,15 @@ up_status up_column_from_host_compact(up_ctx *c, const uint8_t *bytes, up_column
         if (up_status s = scratch_locked(c, sizeof(uint32_t) * (size_t)dst->limbs * (size_t)ld, (void **)&planes)) return s;
     }
     const int nck = (int)std::max<size_t>(1, std::min<size_t>(kIngestChunks, nb / kIngestChunkMin));
-    // the copy stream starts after the caller's prior work (the stage may still be read)
-    CUDA_TRY(cudaEventRecord(c->chunk_ev[0], st));
-    CUDA_TRY(cudaStreamWaitEvent(c->copy_st, c->chunk_ev[0], 0));
+    // rows landing in place (compact column): the copies wait for the caller's
+    // prior work on `stream`, which may still read the column.  Into the ctx
+    // stage they need not: every call that uses the stage synchronises before
+    // returning, so the copies may overlap kernels still queued on `stream`
+    // (e.g. the SUM over the previous chunk of a streamed input)
+    if (dst->layout == UP_LAYOUT_COMPACT) {
+        CUDA_TRY(cudaEventRecord(c->chunk_ev[0], st));
+        CUDA_TRY(cudaStreamWaitEvent(c->copy_st, c->chunk_ev[0], 0));
+    }
     for (int k = 0; k < nck; ++k) {
         // chunk boundaries on 256-row multiples: 4-byte-aligned compact rows for the kernel's word loads
         const long long r0 = (n * k / nck) & ~255ll, r1 = k + 1 == nck ? n : (n * (k + 1) / nck) & ~255ll;

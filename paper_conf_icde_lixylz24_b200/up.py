@@ -180,6 +180,23 @@ class Column:
     def desc(self) -> up_column:
         return up_column(self.n, self.ld, self.p, self.s, self.limbs, self.layout, self.data.data_ptr())
 
+    def rows(self, r0: int, r1: int) -> "Column":
+        """Rows [r0, r1) as a column sharing this one's memory (same ld; r0 a
+        multiple of 4, of 16 for compact rows, keeps the 16-byte alignment)."""
+        if not 0 <= r0 <= r1 <= self.n:
+            raise ValueError("bad row range")
+        v = Column.__new__(Column)
+        v.p, v.s, v.n, v.limbs, v.layout, v.ld = self.p, self.s, r1 - r0, self.limbs, self.layout, self.ld
+        if self.layout == LAYOUT_COMPACT:
+            v.data = self.data[r0 * self.ld:]
+        elif self.layout == LAYOUT_QUADS:
+            v.data = self.data[:, r0:, :]
+        else:
+            v.data = self.data[:, r0:]
+        if v.data.data_ptr() % 16:
+            raise ValueError("row view not 16-byte aligned")
+        return v
+
     @property
     def type(self):
         return (self.p, self.s)
