@@ -1332,7 +1332,9 @@ up_status up_gen_source(const char *variant, const char *expr, const up_column *
     std::string src;
     std::unique_ptr<Node> opt_root = getenv("UP_NO_OPT") ? nullptr : optimize(t.root.get(), t.types);
     const Node *gen_root = opt_root ? opt_root.get() : t.root.get();
-    if (o.sum && max_limbs(gen_root) >= kWideMinLimbs && o.LA <= 512 && !getenv("UP_NO_WIDE"))
+    bool any_compact = false;   // as expr_kernel: the wide regime reads limb planes only
+    for (const ColType &ct : t.types) any_compact = any_compact || ct.Lb > 0 || ct.Q;
+    if (o.sum && !any_compact && max_limbs(gen_root) >= kWideMinLimbs && o.LA <= 512 && !getenv("UP_NO_WIDE"))
         src = gen_wide_sum_kernel(gen_root, t.types, o.LA, info);
     if (src.empty()) src = gen_expr_kernel(gen_root, t.types, o, info);
     if (src.size() + 1 > len) return fail(UP_E_NOMEM, "need %zu bytes", src.size() + 1);
