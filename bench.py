@@ -4,7 +4,9 @@
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C] [--impl up|reference]
 
 Default workload = BASELINE.json configs[1] (the paper's Fig. 1 high-p query):
-SELECT SUM(c1+c2), 10M tuples per GPU, c1 DECIMAL(35,5), c2 DECIMAL(32,2).
+SELECT SUM(c1+c2), 10M tuples per GPU, c1 DECIMAL(35,5), c2 DECIMAL(32,2),
+the columns resident in the paper's compact rows (29 B/row; --layout planes
+for limb planes, 32 B/row).
 Other configs (parity-test cases by default, bench lines on request):
   1  SUM(c1+c2) DECIMAL(17,5)+DECIMAL(14,2), 1M tuples (L2-resident: flushed)
   3  SUM(c1*c2 - c3/c4) DECIMAL(200,50) x4, 12.5M tuples/GPU (100M on 8)
@@ -537,7 +539,7 @@ def main():
     ap.add_argument("--impl", default="up", choices=["up", "reference"])
     ap.add_argument("--layout", default=None, choices=["planes", "compact", "quads"],
                     help="column storage for the expression configs (1-3): limb planes, the paper's compact rows or "
-                         "limb quads (default: planes for 1-2, quads for 3 -- the layout its tensor-core "
+                         "limb quads (default: compact rows for 1-2, quads for 3 -- the layout its tensor-core "
                          "contraction reads straight from TMA)")
     ap.add_argument("--ref-rows", type=int, default=200_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -564,7 +566,14 @@ def main():
         cfg["types"] = [(args.p, s)] * 4
         cfg["name"] = f"cfg3 SUM(c1*c2 - c3/c4) DECIMAL({args.p},{s})"
     if args.layout is None:
-        args.layout = "quads" if cfg["kind"] == "expr" and cfg["types"][0][0] >= 100 else "planes"
+        # expression configs: the paper's compact rows for the narrow columns
+        # (cDecimal, P:L843-873 -- fewer bytes per row than limb planes, read in
+        # place by the fused kernel), limb quads for the wide ones (the tensor
+        # cores' operand layout); modexp / sine read limb planes
+        if cfg["kind"] != "expr":
+            args.layout = "planes"
+        else:
+            args.layout = "quads" if cfg["types"][0][0] >= 100 else "compact"
     if not args.steps:
         args.steps = {"expr": 200, "modexp": 5, "sin": 3}[cfg["kind"]] if cfg["kind"] != "expr" or \
             cfg["types"][0][0] < 100 else 5
