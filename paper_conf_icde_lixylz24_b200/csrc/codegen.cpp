@@ -88,13 +88,22 @@ struct Emitter {
     // when they are the same column)
     std::map<std::pair<int, int>, std::string> wq;   // (column, quad) -> uint4 of this division's window
     std::string top_limb(const Node *n, const std::string &x, int j) {
-        if (!is_lazy(n) || !quad[(size_t)n->col]) return limb(n, x, j);
+        if (!is_lazy(n)) return limb(n, x, j);
+        if (!quad[(size_t)n->col]) {   // plane limb, requested before the decision's branches
+            const std::pair<int, int> key(n->col, 1000000 + j);
+            auto it = wq.find(key);
+            if (it == wq.end()) {
+                std::string v = fresh("w");
+                o << "    const u32 " << v << " = ld_issue1(g" << n->col << " + " << lazy_off(n->col, j) << ");\n";
+                it = wq.emplace(key, v).first;
+            }
+            return it->second;
+        }
         const auto key = std::make_pair(n->col, j >> 2);
         auto it = wq.find(key);
         if (it == wq.end()) {
             std::string v = fresh("q");
-            o << "    const uint4 " << v << " = __ldg(reinterpret_cast<const uint4 *>(g" << n->col << " + (long long)" << (j >> 2)
-              << " * l" << n->col << "));\n";
+            o << "    const uint4 " << v << " = ld_issue4(g" << n->col << " + (long long)" << (j >> 2) << " * l" << n->col << ");\n";
             it = wq.emplace(key, v).first;
         }
         static const char *f[4] = {".x", ".y", ".z", ".w"};
