@@ -181,14 +181,23 @@ class ExprWorkload(Workload):
             mag, neg = gdev.uniform_decimal(self.rows, p, self.args.config, k + 1, row0=self.row0,
                                             nonzero_lead=(k in cfg.get("lead", ())))
             self.raw.append((mag, neg))
-            self.cols.append(ctx.column_from_device_bin(p, s, mag, neg, layout=self.args.layout))
+            self.cols.append(ctx.column_from_device_bin(p, s, mag, neg, layout=self.col_layout(k)))
         ctx.check()
         self.P, self.S, self.LA = ctx.sum_type(cfg["expr"], self.cols, self.n_global)
-        self.e2e_cols = [up.Column(p, s, self.e2e_rows, layout=self.args.layout) for p, s in cfg["types"]]
+        self.e2e_cols = [up.Column(p, s, self.e2e_rows, layout=self.col_layout(k)) for k, (p, s) in enumerate(cfg["types"])]
         # algorithmic bytes per row: the columns as stored -- limb planes (4 B per
         # limb), the paper's compact rows (Lb bytes) or limb quads
         # (16 B per quad, the sign-flag limb and padding included)
-        self.bytes_per_row = sum(_col_bytes(p, self.args.layout) for p, s in cfg["types"])
+        self.bytes_per_row = sum(_col_bytes(p, self.col_layout(k)) for k, (p, s) in enumerate(cfg["types"]))
+
+    def col_layout(self, k):
+        """layout of column k: --layout, or for "mixed" (cfg3's default) limb quads
+        for the product's columns c1, c2 (the tensor cores read them straight
+        from TMA) and limb planes for the division's c3, c4 (fewer bytes beside
+        the concurrent contraction)"""
+        if self.args.layout == "mixed":
+            return "quads" if k < 2 else "planes"
+        return self.args.layout
 
     def kernel(self, out):
         self.ctx.sum_expr(self.cfg["expr"], self.cols, self.n_global, out=out)
@@ -268,7 +277,7 @@ class ExprWorkload(Workload):
         t_tc = self._time(lambda: self.ctx.sum_expr("c1*c2", [c1, c2], self.n_global, out=out))
         t_rest = self._time(lambda: self.ctx.sum_expr("c1/c2", [c3, c4], self.n_global, out=out))
         peak = peaks.get("hbm_gbs", 6650.0)
-        tc_row = _col_bytes(p, self.args.layout)
+        tc_row = _col_bytes(p, self.col_layout(0))
         tc_bytes = 2 * tc_row * self.rows
         ach = tc_bytes / (t_tc / 1e3) / 1e9
         # the rest kernel's arithmetic: the top-limb decision per row (DESIGN §5,
@@ -284,10 +293,10 @@ class ExprWorkload(Workload):
         rest_ach = div_products * self.rows / (t_rest / 1e3)
         return {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
                 "kernel_ms": round(t_tc, 5), "alg_bytes_per_launch": tc_bytes,
-                "alg_unit": f"contraction kernel: c1, c2 as stored ({self.args.layout}) {2 * tc_row} B/row x {self.rows} rows",
+                "alg_unit": f"contraction kernel: c1, c2 as stored ({self.col_layout(0)}) {2 * tc_row} B/row x {self.rows} rows",
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s",
                 "kernels": [
-                    {"kernel": ("k_contract_tq" if self.args.layout == "quads" else "k_contract_tc") +
+                    {"kernel": ("k_contract_tq" if self.col_layout(0) == "quads" else "k_contract_tc") +
                                " (SUM(c1*c2), tcgen05 kind::i8)", "ms": round(t_tc, 5), "bound": "hbm",
                      "alg_bytes": tc_bytes, "achieved_gbs": round(ach, 1), "frac": round(ach / peak, 4)},
                     {"kernel": "upk rest (SUM(-c3/c4), top-limb division)", "ms": round(t_rest, 5), "bound": "alu",
@@ -537,10 +546,10 @@ def main():
     ap.add_argument("--rows", type=int, default=0, help="rows per GPU (default: the config's)")
     ap.add_argument("--global-rows", type=int, default=0, help="total rows, sharded over the GPUs (strong scaling)")
     ap.add_argument("--impl", default="up", choices=["up", "reference"])
-    ap.add_argument("--layout", default=None, choices=["planes", "compact", "quads"],
+    ap.add_argument("--layout", default=None, choices=["planes", "compact", "quads", "mixed"],
                     help="column storage for the expression configs (1-3): limb planes, the paper's compact rows or "
-                         "limb quads (default: compact rows for 1-2, quads for 3 -- the layout its tensor-core "
-                         "contraction reads straight from TMA)")
+                         "limb quads, or mixed (cfg3: quads for the product's c1, c2, planes for c3, c4); default: "
+                         "compact rows for 1-2, mixed for 3")
     ap.add_argument("--ref-rows", type=int, default=200_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-pipelined", action="store_true",
@@ -568,12 +577,13 @@ def main():
     if args.layout is None:
         # expression configs: the paper's compact rows for the narrow columns
         # (cDecimal, P:L843-873 -- fewer bytes per row than limb planes, read in
-        # place by the fused kernel), limb quads for the wide ones (the tensor
-        # cores' operand layout); modexp / sine read limb planes
+        # place by the fused kernel); for cfg3 limb quads for the product's
+        # columns (the tensor cores' operand layout) and limb planes for the
+        # division's; modexp / sine read limb planes
         if cfg["kind"] != "expr":
             args.layout = "planes"
         else:
-            args.layout = "quads" if cfg["types"][0][0] >= 100 else "compact"
+            args.layout = "mixed" if cfg["types"][0][0] >= 100 else "compact"
     if not args.steps:
         args.steps = {"expr": 200, "modexp": 5, "sin": 3}[cfg["kind"]] if cfg["kind"] != "expr" or \
             cfg["types"][0][0] < 100 else 5

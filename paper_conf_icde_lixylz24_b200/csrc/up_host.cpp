@@ -182,6 +182,12 @@ struct up_ctx {
     // chunk k+1 overlaps the conversion / range check of chunk k
     cudaStream_t copy_st = nullptr;
     cudaEvent_t chunk_ev[kIngestChunks] = {};
+    // split SUMs over quad columns: the tensor-core contraction on a side stream
+    // (own workspace + ticket) beside the rest kernel on the caller's stream
+    cudaStream_t side = nullptr, side_rest = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_join_rest = nullptr;
+    unsigned long long *d_ws2 = nullptr;
+    uint32_t *d_ticket2 = nullptr;
     std::mutex mu;
 };
 
@@ -376,13 +382,13 @@ std::string key_of(const char *tag, const char *expr, const up_column *cols, int
     return k;
 }
 
-up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream_t st) {
+up_status launch(up_ctx *c, JitKernel *k, up_kparams &P, long long n, cudaStream_t st, bool allow_pdl = true) {
     long long per_block = k->rows_per_block > 0 ? k->rows_per_block : (long long)k->threads * k->rows_per_thread;
     long long want = (n + per_block - 1) / per_block;
     long long cap = (long long)k->blocks_per_sm * c->num_sms;
     int grid = (int)std::max(1ll, std::min(want, cap));
     void *args[] = {&P};
-    if (k->pdl && c->pipelined) {
+    if (k->pdl && c->pipelined && allow_pdl) {
         CUlaunchAttribute at[1];
         at[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
         at[0].value.programmaticStreamSerializationAllowed = 1;
@@ -539,6 +545,13 @@ up_status up_ctx_destroy(up_ctx *c) {
     if (c->d_stage) cudaFree(c->d_stage);
     for (cudaEvent_t e : c->chunk_ev) if (e) cudaEventDestroy(e);
     if (c->copy_st) cudaStreamDestroy(c->copy_st);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
+    if (c->ev_join_rest) cudaEventDestroy(c->ev_join_rest);
+    if (c->side) cudaStreamDestroy(c->side);
+    if (c->side_rest) cudaStreamDestroy(c->side_rest);
+    if (c->d_ws2) cudaFree(c->d_ws2);
+    if (c->d_ticket2) cudaFree(c->d_ticket2);
     if (c->d_scratch) cudaFree(c->d_scratch);
     if (c->d_parts) cudaFree(c->d_parts);
     delete c;
@@ -988,7 +1001,12 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             const int T = (int)pl.prods.size() + (pl.rest_kernel ? 1 : 0);
             const size_t need = (size_t)T * (size_t)LAs;
             if (need > c->parts_words) {
-                if (c->d_parts) { CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream)); CUDA_TRY(cudaFree(c->d_parts)); }
+                if (c->d_parts) {
+                    CUDA_TRY(cudaStreamSynchronize((cudaStream_t)stream));
+                    if (c->side) CUDA_TRY(cudaStreamSynchronize(c->side));
+                    if (c->side_rest) CUDA_TRY(cudaStreamSynchronize(c->side_rest));
+                    CUDA_TRY(cudaFree(c->d_parts));
+                }
                 CUDA_TRY(cudaMalloc(&c->d_parts, sizeof(uint32_t) * need * 2));
                 c->parts_words = need * 2;
             }
@@ -997,14 +1015,52 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             P.ws = c->d_ws;
             P.ticket = c->d_ticket;
             P.flags = c->d_flags;
+            // quad contractions + a rest kernel: the contraction (6 warps and its
+            // shared-memory stages, HBM-bound) and the integer-bound rest kernel
+            // run side by side on two ctx streams forked from the caller's stream
+            // (the contraction with its own workspace and ticket), joined before
+            // the combine.  Both off the caller's stream: on the legacy default
+            // stream the pair overlapped less (0.77 vs 0.68 ms, profiles/r02_s66).
+            // UP_SERIAL_SPLIT: everything on the caller's stream, back to back.
+            // Only for contractions of at most two roles per row block (p <= ~600):
+            // with more, the contraction's own MMA / copy overlap is the limit and
+            // sharing the SMs slows it more than the division gains (p = 1000:
+            // 3.76 vs 3.56 ms back to back, profiles/r02_s67)
+            bool overlap = pl.rest_kernel != nullptr && !getenv("UP_SERIAL_SPLIT");
+            for (size_t q = 0; q < pl.prods.size() && overlap; ++q) {
+                const int ga = (cols[pl.prods[q].col_a].limbs + 4) / 4, gb = (cols[pl.prods[q].col_b].limbs + 4) / 4;
+                overlap = !pl.cc_kernels[q] && cols[pl.prods[q].col_a].layout == UP_LAYOUT_QUADS &&
+                          ((ga + 7) / 8) * ((gb + 31) / 32) <= 2;
+            }
+            cudaStream_t tcs = (cudaStream_t)stream;
+            unsigned long long *tws = c->d_ws;
+            uint32_t *ttk = c->d_ticket;
+            if (overlap) {
+                if (!c->side) {
+                    CUDA_TRY(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
+                    CUDA_TRY(cudaStreamCreateWithFlags(&c->side_rest, cudaStreamNonBlocking));
+                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+                    CUDA_TRY(cudaEventCreateWithFlags(&c->ev_join_rest, cudaEventDisableTiming));
+                    CUDA_TRY(cudaMalloc(&c->d_ws2, sizeof(unsigned long long) * 2 * 1024));
+                    CUDA_TRY(cudaMemset(c->d_ws2, 0, sizeof(unsigned long long) * 2 * 1024));
+                    CUDA_TRY(cudaMalloc(&c->d_ticket2, 64));
+                    CUDA_TRY(cudaMemset(c->d_ticket2, 0, 64));
+                    CUDA_TRY(cudaDeviceSynchronize());
+                }
+                CUDA_TRY(cudaEventRecord(c->ev_fork, (cudaStream_t)stream));
+                CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+                CUDA_TRY(cudaStreamWaitEvent(c->side_rest, c->ev_fork, 0));
+                tcs = c->side; tws = c->d_ws2; ttk = c->d_ticket2;
+            }
             int ti = 0;
             for (size_t q = 0; q < pl.prods.size(); ++q) {
                 const SplitTerm &st = pl.prods[q];
                 const up_column &ca = cols[st.col_a], &cb = cols[st.col_b];
                 if (!pl.cc_kernels[q]) {
                     auto tc = ca.layout == UP_LAYOUT_QUADS ? upk_launch_contract_tq : upk_launch_contract_tc;
-                    CUDA_TRY(tc(ca.data, ca.ld, ca.limbs, cb.data, cb.ld, cb.limbs, cols[0].n, st.sign, c->d_ws, c->d_ticket,
-                                c->d_parts + (size_t)ti++ * LAs, LAs, c->num_sms, (cudaStream_t)stream));
+                    CUDA_TRY(tc(ca.data, ca.ld, ca.limbs, cb.data, cb.ld, cb.limbs, cols[0].n, st.sign, tws, ttk,
+                                c->d_parts + (size_t)ti++ * LAs, LAs, c->num_sms, tcs));
                     c->launches++;
                     continue;
                 }
@@ -1013,7 +1069,15 @@ up_status up_sum_expr(up_ctx *c, const char *expr, const up_column *cols, int nc
             }
             if (pl.rest_kernel) {
                 P.result = c->d_parts + (size_t)ti++ * LAs;
-                if (up_status s = launch(c, pl.rest_kernel, P, P.n, (cudaStream_t)stream)) return s;
+                // (no programmatic launch beside the contraction: measured slower, r02_s67)
+                if (up_status s = launch(c, pl.rest_kernel, P, P.n, overlap ? c->side_rest : (cudaStream_t)stream, !overlap))
+                    return s;
+            }
+            if (overlap) {
+                CUDA_TRY(cudaEventRecord(c->ev_join, c->side));
+                CUDA_TRY(cudaEventRecord(c->ev_join_rest, c->side_rest));
+                CUDA_TRY(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_join, 0));
+                CUDA_TRY(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_join_rest, 0));
             }
             if (pl.rest_kernel && pl.rest_scale > 0) {
                 const uint32_t *d_sc = nullptr;

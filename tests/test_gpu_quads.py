@@ -114,16 +114,23 @@ def test_quad_contraction_empty():
 CFG3 = [(200, 50), (500, 75), (1000, 100)]
 
 
+@pytest.mark.parametrize("lays", ["qqqq", "qqpp"])
+@pytest.mark.parametrize("serial", [False, True], ids=["side-stream", "serial"])
 @pytest.mark.parametrize("ps", CFG3, ids=lambda t: f"p{t[0]}")
 @pytest.mark.parametrize("n", [1, 1000, 4099])
-def test_cfg3_sum_quads(ps, n):
-    """cfg3's SUM(c1*c2 - c3/c4) over quad columns (tensor-core contraction +
-    the fused top-limb division reading quads) == the oracle"""
+def test_cfg3_sum_quads(ps, n, serial, lays, monkeypatch):
+    """cfg3's SUM(c1*c2 - c3/c4) with c1, c2 in quads (tensor-core contraction
+    on the ctx side stream beside the fused top-limb division, or both on one
+    stream with UP_SERIAL_SPLIT; c3, c4 quads or planes -- the bench's "mixed")
+    == the oracle"""
+    if serial:
+        monkeypatch.setenv("UP_SERIAL_SPLIT", "1")
     types = [ps] * 4
     host = G.gen_cols(n, types, config=3, nonzero_lead_cols=(3,))
     want, P, S = oracle.eval_sum("c1*c2 - c3/c4", G.to_oracle(host, types), n=n, threads=8)
     c = G.ctx()
-    gcols = [c.column_from_host_bin(p, s, m, g, layout="quads") for (m, g), (p, s) in zip(host, types)]
+    layout = {"q": "quads", "p": "planes"}
+    gcols = [c.column_from_host_bin(p, s, m, g, layout=layout[lays[k]]) for k, ((m, g), (p, s)) in enumerate(zip(host, types))]
     got, gP, gS = G.gpu_sum_string("c1*c2 - c3/c4", gcols)
     assert (gP, gS) == (P, S)
     assert got == want

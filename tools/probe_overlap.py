@@ -61,6 +61,12 @@ def main():
     def split():
         c1.sum_expr("c1*c2 - c3/c4", cols, n, out=o3)
 
+    def split_on_stream():   # the library's split, called on a created (non-legacy) stream
+        cur = torch.cuda.current_stream()
+        s2.wait_stream(cur)
+        c1.sum_expr("c1*c2 - c3/c4", cols, n, out=o3, stream=s2)
+        cur.wait_stream(s2)
+
     def t(fn):
         for _ in range(3):
             fn()
@@ -74,7 +80,7 @@ def main():
         return round(e0.elapsed_time(e1) / a.reps, 4)
 
     r = {"p": a.p, "rows": n, "rest_layout": a.rest_layout, "tc_ms": t(tc), "rest_ms": t(rest), "serial_ms": t(both_serial),
-         "two_streams_ms": t(both_streams), "split_step_ms": t(split)}
+         "two_streams_ms": t(both_streams), "split_step_ms": t(split), "split_on_stream_ms": t(split_on_stream)}
     print(json.dumps(r))
 
 
