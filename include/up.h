@@ -181,7 +181,13 @@ up_status up_eval_expr(up_ctx *ctx, const char *expr, const up_column *cols, int
  * The result type is DECIMAL(p_expr + ceil(log10 n_global), s_expr) with
  * LA = up_limbs(that p) limbs (query with up_sum_type).  d_partial receives LA
  * two's-complement limbs (device).  n_global = rows over all shards (typing
- * only; 0 means cols[0].n).  One kernel launch.
+ * only; 0 means cols[0].n).  One kernel launch -- except when a top-level
+ * product of two wide columns is split off (SUM is linear): its tensor-core
+ * contraction, the fused kernel for the rest of the expression and an exact
+ * combine kernel; over limb-quad columns the contraction and the rest run on
+ * two ctx-owned streams forked from `stream` and joined back into it before
+ * the combine (the call stays ordered on `stream`; UP_SERIAL_SPLIT keeps
+ * everything on `stream`).
  */
 up_status up_sum_type(up_ctx *ctx, const char *expr, const up_column *cols, int ncols,
                       int64_t n_global, int32_t *p, int32_t *s, int32_t *la);
