@@ -136,7 +136,7 @@ def test_quad_layout_kernels_compile_for_sm100a(variant, expr, types, layouts, t
     them with 16-byte loads and compile for sm_100a; the division's decision
     window loads whole quads and its full-division fallback is out of line"""
     src = up.gen_source(variant, expr, types, 1_000_000, layouts=layouts)
-    assert "ld_quads<" in src or "reinterpret_cast<const uint4 *>(g" in src
+    assert "ld_quads<" in src or "ld_issue4(g" in src
     if expr == "c1/c2":   # both division operands are columns read lazily: fallback out of line
         assert "__noinline__" in src and "div_top_decide<" in src
     log = up.nvrtc_compile(src, str(tmp_path / "q.cubin"))
